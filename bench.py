@@ -1,0 +1,392 @@
+#!/usr/bin/env python
+"""IDG gridding + degridding throughput on B200 (BASELINE.json metric), one JSON line on rank 0.
+
+A step = one pass of the hot path over the LOFAR-shaped data set (BASELINE.json configs[1]):
+    grid(visibilities) -> [N>1: NCCL reduce of the uv-grid to rank 0 -> broadcast] -> degrid(grid)
+The plan (host, built once per observation, "before any execution") is built before the timed
+region and reported separately as plan_s.  value = visibilities per step / step time (MVis/s),
+whole job; with N GPUs the baselines are split into N contiguous shards (strong scaling).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config lofar] [--impl ours|reference]
+
+--impl reference times the fp64 CPU oracle (oracle/, the correctness reference) on the host cores, on a
+bounded sample of the same workload per step; under torchrun only rank 0 runs it.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import idgsynth  # noqa: E402
+
+BASELINE = json.load(open(os.path.join(ROOT, "BASELINE.json")))
+METRIC = BASELINE["metric"]
+OPS_PER_PAIR = 36        # 17 FMA (2 ops) + sin + cos per (pixel, visibility) pair
+CONFIG_NAMES = {"tiny": 0, "lofar": 1, "lofar_dde": 2, "ska": 3, "predict": 4}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ------------------------------------------------------------------------------------------------
+# clocks during the timed region (NVML = what nvidia-smi reads)
+# ------------------------------------------------------------------------------------------------
+class ClockSampler:
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, torch_device: int, period_s: float = 0.1):
+        self.period = period_s
+        self.samples, self.reasons = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._h = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            import torch
+            p = torch.cuda.get_device_properties(torch_device)
+            bus = f"{p.pci_domain_id:08x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+            self._h = pynvml.nvmlDeviceGetHandleByPciBusId(bus.encode())
+            self._nvml = pynvml
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+        except Exception as e:  # pragma: no cover
+            log(f"[bench] NVML unavailable: {e}")
+
+    def _run(self):
+        n = self._nvml
+        while not self._stop.is_set():
+            try:
+                self.samples.append(n.nvmlDeviceGetClockInfo(self._h, n.NVML_CLOCK_SM))
+                mask = n.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                for bit, name in self.REASONS.items():
+                    if mask & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            self._stop.wait(self.period)
+
+    def __enter__(self):
+        if self._h is not None:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *exc):
+        self._stop.set()
+        if self._h is not None:
+            self._t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------------------------------------
+# distributed plumbing
+# ------------------------------------------------------------------------------------------------
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def shard_range(nbl: int, rank: int, world: int):
+    """Contiguous baseline shard of rank r (work per baseline = its visibilities x N~^2)."""
+    b0 = (nbl * rank) // world
+    b1 = (nbl * (rank + 1)) // world
+    return b0, b1
+
+
+def workload_description(name):
+    obs_cfg = idgsynth.CONFIGS[name]
+    return (f"{BASELINE['configs'][CONFIG_NAMES[name]]} | synthetic: {obs_cfg['nr_stations']} stations, "
+            f"T={obs_cfg['T']}, C={obs_cfg['C']}, N~={obs_cfg['Ns']}, N={obs_cfg['N']}, K={obs_cfg['K']}, "
+            f"T~max={obs_cfg['Tmax']}, A-terms={obs_cfg['aterms']} (slots of {obs_cfg['slot']})")
+
+
+# ------------------------------------------------------------------------------------------------
+# CPU oracle (cpu_baseline / --impl reference)
+# ------------------------------------------------------------------------------------------------
+def oracle_sample(obs, target_s: float):
+    """Choose a deterministic sample (first baselines x all timesteps) worth ~target_s of oracle time."""
+    import oracle
+    probe = obs.subset(nr_baselines=1, nr_timesteps=min(obs.nr_timesteps, 16 * obs.max_timesteps_per_subgrid))
+    t = time_oracle_step(probe)[0]
+    per_vis = t / max(1, probe.nr_visibilities)
+    want_vis = target_s / max(per_vis, 1e-12)
+    nt = obs.nr_timesteps
+    nb = max(1, min(obs.nr_baselines, int(want_vis // (nt * obs.nr_channels))))
+    if nb == 1 and want_vis < nt * obs.nr_channels:
+        nt = max(obs.max_timesteps_per_subgrid, int(want_vis // obs.nr_channels))
+        nt = min(nt, obs.nr_timesteps)
+    return obs.subset(nr_baselines=nb, nr_timesteps=nt)
+
+
+def time_oracle_step(sample):
+    import oracle
+    vis = idgsynth.make_visibilities(sample)
+    aterms = idgsynth.make_aterms(sample)
+    taper = idgsynth.make_taper(sample.subgrid_size)
+    items, _ = oracle.plan(sample)
+    t0 = time.perf_counter()
+    g = oracle.grid(sample, items, vis, aterms, taper)
+    t1 = time.perf_counter()
+    oracle.degrid(sample, items, g.astype(np.complex64), aterms, taper)
+    t2 = time.perf_counter()
+    nvis = int(np.sum(items["nr_timesteps"].astype(np.int64) * (items["channel_end"] - items["channel_begin"])))
+    return t2 - t0, nvis, t1 - t0, t2 - t1
+
+
+def cpu_baseline(obs, target_s=15.0):
+    import oracle
+    sample = oracle_sample(obs, target_s)
+    dt, nvis, tg, td = time_oracle_step(sample)
+    return {"value": nvis / dt / 1e6, "unit": "MVis/s", "cores": oracle.max_threads(), "kind": "oracle",
+            "sample": f"{sample.nr_baselines} baselines x {sample.nr_timesteps} timesteps x "
+                      f"{sample.nr_channels} channels of '{obs.name}' ({nvis} visibilities), grid {tg:.2f} s + "
+                      f"degrid {td:.2f} s, fp64 C + OpenMP"}
+
+
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    import oracle
+    obs = idgsynth.make_observation(args.config)
+    sample = oracle_sample(obs, args.reference_step_s)
+    for _ in range(args.warmup):
+        time_oracle_step(sample)
+    times, nvis = [], 0
+    for _ in range(args.steps):
+        dt, nvis, _, _ = time_oracle_step(sample)
+        times.append(dt)
+    total = sum(times)
+    value = nvis * args.steps / total / 1e6
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "MVis/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": workload_description(args.config), "sample_baselines": sample.nr_baselines,
+                       "sample_timesteps": sample.nr_timesteps, "parallelism": "host OpenMP"},
+            "cpu_baseline": {"value": value, "unit": "MVis/s", "cores": oracle.max_threads(), "kind": "oracle",
+                             "sample": f"{sample.nr_baselines} baselines x {sample.nr_timesteps} timesteps x "
+                                       f"{sample.nr_channels} channels ({nvis} visibilities) per step"},
+            "e2e": {"value": value, "unit": "MVis/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------------------------
+# our arm
+# ------------------------------------------------------------------------------------------------
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_veenboerpr17_b200 as idg
+    from paper_conf_ipps_veenboerpr17_b200 import _build
+    if not os.path.exists(_build.LIB):
+        _build.build()
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    full = idgsynth.make_observation(args.config)
+    b0, b1 = shard_range(full.nr_baselines, rank, world)
+    obs = full.subset(nr_baselines=b1 - b0, baseline_begin=b0)
+    t0 = time.perf_counter()
+    plan = idg.Plan.from_observation(obs)
+    plan_s = time.perf_counter() - t0
+    st = plan.stats()
+    pairs = st["nr_pairs"]
+    nvis_rank = st["nr_vis_assigned"]
+
+    aterms = idgsynth.make_aterms(obs)
+    taper = idgsynth.make_taper(obs.subgrid_size)
+    uvw_d = torch.from_numpy(obs.uvw).to(dev)
+    at_d = torch.from_numpy(aterms).to(dev)
+    tp_d = torch.from_numpy(taper).to(dev)
+    vis_d = idgsynth.torch_visibilities(obs, dev, seed_offset=11 + b0)
+    out_d = torch.empty_like(vis_d)
+    N = obs.grid_size
+    grid_d = torch.zeros((4, N, N), dtype=torch.complex64, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    def step(vis_in, vis_out):
+        grid_d.zero_()
+        idg.grid(plan, vis_in, uvw_d, at_d, tp_d, grid_d)
+        if world > 1:
+            dist.reduce(grid_d, dst=0)          # a5 across ranks: sum of the per-shard uv-grids
+            dist.broadcast(grid_d, src=0)       # the model grid for degridding (here: the gridded data)
+        idg.degrid(plan, grid_d, uvw_d, at_d, tp_d, vis_out)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+
+    for _ in range(args.warmup):
+        step(vis_d, out_d)
+    barrier()
+
+    # ---- timed region: device-resident inputs -------------------------------------------------
+    idg.profiling_reset()
+    idg.profiling_enable(True)
+    launches0 = idg.launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clocks:
+        barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            step(vis_d, out_d)
+        ev1.record(stream)
+        barrier()
+    idg.profiling_enable(False)
+    gpu_launches = idg.launch_count() - launches0
+    kern = idg.profiling_read()
+    ms = ev0.elapsed_time(ev1)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    nvis_t = torch.tensor([nvis_rank], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(nvis_t)
+    nvis_total = float(nvis_t.item())
+    value = nvis_total * args.steps / (ms_max * 1e-3) / 1e6
+
+    # ---- e2e: host buffers through the public API (H2D of inputs + D2H of the prediction) --------
+    e2e = None
+    if not args.no_e2e:
+        vis_h = torch.empty(vis_d.shape, dtype=vis_d.dtype, pin_memory=True)
+        vis_h.copy_(vis_d)
+        out_h = torch.empty_like(vis_h, pin_memory=True)
+        uvw_h = torch.from_numpy(obs.uvw).pin_memory()
+
+        def e2e_step():
+            uvw_d.copy_(uvw_h, non_blocking=True)
+            vis_d.copy_(vis_h, non_blocking=True)
+            step(vis_d, out_d)
+            out_h.copy_(out_d, non_blocking=True)
+
+        e2e_step()
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ksteps = max(1, min(args.steps, args.e2e_steps))
+        e0.record(stream)
+        for _ in range(ksteps):
+            e2e_step()
+        e1.record(stream)
+        barrier()
+        te = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e = {"value": nvis_total * ksteps / (float(te.item()) * 1e-3) / 1e6, "unit": "MVis/s",
+               "h2d_bytes_per_step": int(vis_h.numel() * 8 + uvw_h.numel() * 4),
+               "d2h_bytes_per_step": int(out_h.numel() * 8), "steps": ksteps}
+        del vis_h, out_h
+
+    # ---- roofline: paper's modified roofline = FMA:sincos benchmark at rho = 17, same process -----
+    rho_ops, _ = idg.rho_benchmark(17, args.rho_iterations)
+    rho_sweep = {}
+    if args.rho_sweep:
+        for r in (1, 2, 4, 8, 12, 16, 17, 24, 32, 64):
+            rho_sweep[str(r)] = idg.rho_benchmark(r, args.rho_iterations)[0] / 1e12
+    per_kernel = {}
+    for name in ("gridder", "degridder"):
+        k = kern.get(name)
+        if not k:
+            continue
+        avg_ms = k["total_ms"] / k["launches"]
+        achieved = OPS_PER_PAIR * pairs / (avg_ms * 1e-3) / 1e12
+        per_kernel[name] = {"launches": k["launches"], "avg_ms": avg_ms, "TOps_s": achieved,
+                            "frac": achieved / (rho_ops / 1e12),
+                            "share_of_step": k["total_ms"] / (ms / 1.0)}
+    dominant = max(per_kernel, key=lambda n: per_kernel[n]["avg_ms"]) if per_kernel else None
+    sm_mhz = clocks.summary()["sm_mhz"] or 1965
+    # theoretical issue-bound peak: 4 SMSPs x 32 lanes / 20 issue slots per pair (18 FP32 + 2 MUFU)
+    theo = 148 * 128 / 20 * OPS_PER_PAIR * sm_mhz * 1e6 / 1e12
+    traffic = None
+    prof_json = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if dominant and os.path.exists(prof_json):
+        try:
+            traffic = json.load(open(prof_json)).get(args.config, {}).get(dominant, {}).get("dram_bytes")
+        except Exception:
+            traffic = None
+    roofline = None
+    if dominant:
+        roofline = {"bound": "alu", "kernel": dominant, "achieved": per_kernel[dominant]["TOps_s"],
+                    "peak": rho_ops / 1e12, "unit": "TOps/s", "frac": per_kernel[dominant]["frac"],
+                    "traffic": traffic,
+                    "peak_source": "measured rho=17 FMA:sincos benchmark in this process (P:276-290)",
+                    "peak_theoretical_issue_bound": theo, "ops_per_pair": OPS_PER_PAIR,
+                    "pairs_per_launch": pairs}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return 0
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(full, args.cpu_baseline_s)
+    line = {
+        "metric": METRIC, "value": value, "unit": "MVis/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": workload_description(args.config), "visibilities": int(nvis_total),
+                   "subgrids_rank0": st["nr_subgrids"], "pairs_rank0": pairs,
+                   "parallelism": f"baseline shards x{world}" + (" + NCCL reduce/broadcast" if world > 1 else ""),
+                   "l2": "inputs larger than L2 (visibilities 4 GB/step)"},
+        "grid_mvis_s": (nvis_rank / (per_kernel["gridder"]["avg_ms"] * 1e-3) / 1e6) if "gridder" in per_kernel else None,
+        "degrid_mvis_s": (nvis_rank / (per_kernel["degridder"]["avg_ms"] * 1e-3) / 1e6) if "degridder" in per_kernel else None,
+        "plan_s": plan_s, "clocks": clocks.summary(), "e2e": e2e, "gpu_launches": gpu_launches,
+        "roofline": roofline, "kernels": per_kernel, "rho_sweep_TOps_s": rho_sweep or None,
+        "cpu_baseline": cpu,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="lofar", choices=sorted(CONFIG_NAMES))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-baseline-s", type=float, default=15.0)
+    ap.add_argument("--reference-step-s", type=float, default=8.0)
+    ap.add_argument("--rho-iterations", type=int, default=2048)
+    ap.add_argument("--rho-sweep", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        log("[bench] warmup < 3 violates the timing rules; using 3")
+        args.warmup = 3
+    return run_reference(args) if args.impl == "reference" else run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

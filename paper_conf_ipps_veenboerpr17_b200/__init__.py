@@ -1,0 +1,11 @@
+"""B200-native (sm_100a) Image-Domain Gridding hot path: plan / grid / degrid behind a C ABI.
+
+Veenboer, Petschow, Romein, "Image-Domain Gridding on Graphics Processors", IPDPS 2017.
+The product is libidg_b200.so (include/idg.h); this package is its ctypes binding plus the
+multi-GPU sharding glue (torch.distributed, NCCL).  No CPU fallback exists.
+"""
+from .idg import (IDGError, METADATA_DTYPE, Plan, degrid, grid, launch_count, lib, profiling_enable,
+                  profiling_read, profiling_reset, rho_benchmark)
+
+__all__ = ["IDGError", "METADATA_DTYPE", "Plan", "degrid", "grid", "launch_count", "lib", "profiling_enable",
+           "profiling_read", "profiling_reset", "rho_benchmark"]

@@ -1,0 +1,453 @@
+// idg_api.cpp -- the C ABI of include/idg.h: validation, plan object, lazy device copies, kernel
+// launches, profiling.  No C++ exception crosses the ABI; errors map to idg_status and a
+// thread-local message (idg_last_error).
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <new>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "idg_internal.h"
+
+namespace {
+
+thread_local std::string g_last_error;
+
+idg_status fail(idg_status st, const std::string &msg) {
+    g_last_error = msg;
+    return st;
+}
+
+idg_status cuda_fail(cudaError_t e, const char *what) {
+    return fail(IDG_ERR_CUDA, std::string(what) + ": " + cudaGetErrorName(e) + " (" +
+                                  cudaGetErrorString(e) + ")");
+}
+
+std::atomic<int64_t> g_launches{0};
+
+struct ProfileRecord {
+    std::string name;
+    cudaEvent_t e0, e1;
+};
+std::mutex g_prof_mu;
+std::atomic<bool> g_prof_enabled{false};
+std::vector<ProfileRecord> g_prof_pending;
+std::map<std::string, std::pair<int64_t, double>> g_prof_totals;
+
+struct DeviceCopy {
+    idg_metadata *items = nullptr;
+    int32_t *order = nullptr;
+    int32_t *baselines = nullptr;
+    double *frequencies = nullptr;
+};
+
+bool supported_subgrid(int32_t n) { return n == 16 || n == 24 || n == 32; }
+
+}  // namespace
+
+struct idg_plan {
+    idg_plan_params params{};
+    int32_t nr_stations = 0, nr_baselines = 0, nr_timesteps = 0, nr_channels = 0;
+    int32_t nr_aterm_slots = 0;
+    std::vector<int32_t> baselines;  // [nbl][2]
+    std::vector<double> frequencies;
+    std::vector<idg_metadata> items;
+    std::vector<int32_t> order;      // launch order: largest T~ C~ first (tail balance)
+    int64_t nr_vis_assigned = 0, nr_vis_dropped = 0, nr_pairs = 0;
+    int32_t max_channels_in_item = 0;
+    int32_t degridder_v = 1;
+    mutable std::mutex mu;
+    mutable std::map<int, DeviceCopy> device;
+
+    ~idg_plan() {
+        for (auto &kv : device) {
+            int prev = -1;
+            cudaGetDevice(&prev);
+            cudaSetDevice(kv.first);
+            cudaFree(kv.second.items);
+            cudaFree(kv.second.order);
+            cudaFree(kv.second.baselines);
+            cudaFree(kv.second.frequencies);
+            if (prev >= 0) cudaSetDevice(prev);
+        }
+    }
+
+    // Device copy of the plan on the current device, made on first use (thread-safe).
+    idg_status device_copy(const DeviceCopy **out) const {
+        int dev = -1;
+        cudaError_t e = cudaGetDevice(&dev);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+        std::lock_guard<std::mutex> lock(mu);
+        auto it = device.find(dev);
+        if (it != device.end()) {
+            *out = &it->second;
+            return IDG_OK;
+        }
+        cudaDeviceProp prop;
+        e = cudaGetDeviceProperties(&prop, dev);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceProperties");
+        if (prop.major != 10 || prop.minor != 0)
+            return fail(IDG_ERR_UNSUPPORTED, std::string("libidg_b200 is built for sm_100a only; device ") +
+                                                 prop.name + " is sm_" + std::to_string(prop.major) +
+                                                 std::to_string(prop.minor));
+        DeviceCopy dc;
+        const size_t ni = std::max<size_t>(1, items.size());
+        if ((e = cudaMalloc(&dc.items, ni * sizeof(idg_metadata))) != cudaSuccess ||
+            (e = cudaMalloc(&dc.order, ni * sizeof(int32_t))) != cudaSuccess ||
+            (e = cudaMalloc(&dc.baselines, std::max<size_t>(2, baselines.size()) * 4)) != cudaSuccess ||
+            (e = cudaMalloc(&dc.frequencies, frequencies.size() * 8)) != cudaSuccess) {
+            cudaFree(dc.items); cudaFree(dc.order); cudaFree(dc.baselines); cudaFree(dc.frequencies);
+            return e == cudaErrorMemoryAllocation ? fail(IDG_ERR_OUT_OF_MEMORY, "plan device copy")
+                                                  : cuda_fail(e, "cudaMalloc(plan)");
+        }
+        if (!items.empty()) {
+            cudaMemcpy(dc.items, items.data(), items.size() * sizeof(idg_metadata), cudaMemcpyHostToDevice);
+            cudaMemcpy(dc.order, order.data(), order.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
+        }
+        if (!baselines.empty())
+            cudaMemcpy(dc.baselines, baselines.data(), baselines.size() * 4, cudaMemcpyHostToDevice);
+        e = cudaMemcpy(dc.frequencies, frequencies.data(), frequencies.size() * 8, cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy(plan)");
+        auto res = device.emplace(dev, dc);
+        *out = &res.first->second;
+        return IDG_OK;
+    }
+};
+
+namespace idg {
+
+LaunchScope::LaunchScope(const char *n, cudaStream_t s) : name(n), stream(s) {
+    g_launches.fetch_add(1);
+    if (g_prof_enabled.load()) {
+        cudaEventCreate(&e0);
+        cudaEventCreate(&e1);
+        cudaEventRecord(e0, stream);
+    }
+}
+
+LaunchScope::~LaunchScope() {
+    if (e0) {
+        cudaEventRecord(e1, stream);
+        std::lock_guard<std::mutex> lock(g_prof_mu);
+        g_prof_pending.push_back({name, e0, e1});
+    }
+}
+
+}  // namespace idg
+
+namespace {
+
+idg_status validate_params(const idg_plan_params *p) {
+    if (!p) return fail(IDG_ERR_INVALID_ARG, "params is NULL");
+    if (!supported_subgrid(p->subgrid_size))
+        return fail(IDG_ERR_UNSUPPORTED, "subgrid_size must be 16, 24 or 32 (got " +
+                                             std::to_string(p->subgrid_size) + ")");
+    if (p->grid_size < 2 * p->subgrid_size || p->grid_size % 2 != 0 || p->grid_size > (1 << 16))
+        return fail(IDG_ERR_INVALID_ARG, "grid_size must be even, >= 2*subgrid_size and <= 65536");
+    if (!(p->image_size > 0.0) || !std::isfinite(p->image_size) || p->image_size >= 2.0)
+        return fail(IDG_ERR_INVALID_ARG, "image_size must be in (0, 2)");
+    if (p->kernel_size < 0 || p->kernel_size >= p->subgrid_size)
+        return fail(IDG_ERR_INVALID_ARG, "kernel_size must be in [0, subgrid_size)");
+    if (p->max_timesteps_per_subgrid < 1)
+        return fail(IDG_ERR_INVALID_ARG, "max_timesteps_per_subgrid must be >= 1");
+    if (p->max_channels_per_subgrid < 0)
+        return fail(IDG_ERR_INVALID_ARG, "max_channels_per_subgrid must be >= 0");
+    if (!std::isfinite(p->w_offset)) return fail(IDG_ERR_INVALID_ARG, "w_offset is not finite");
+    return IDG_OK;
+}
+
+idg_status validate_call(const idg_plan *plan, const void *a, const void *b, const void *c,
+                         const void *d, const void *e) {
+    if (!plan) return fail(IDG_ERR_INVALID_ARG, "plan is NULL");
+    if (plan->items.empty()) return IDG_OK;
+    if (!a || !b || !c || !d || !e) return fail(IDG_ERR_INVALID_ARG, "NULL device pointer");
+    return IDG_OK;
+}
+
+idg::KernelArgs make_args(const idg_plan *plan, const DeviceCopy *dc, const float *d_uvw,
+                          const void *d_aterms, const float *d_taper, void *d_vis, void *d_grid) {
+    idg::KernelArgs a{};
+    const auto &p = plan->params;
+    a.subgrid_size = p.subgrid_size;
+    a.grid_size = p.grid_size;
+    a.cell_l = float(p.image_size / p.subgrid_size);
+    a.inv_image_size = 1.0 / p.image_size;
+    a.w_offset = p.w_offset;
+    a.nr_stations = plan->nr_stations;
+    a.nr_baselines = plan->nr_baselines;
+    a.nr_timesteps = plan->nr_timesteps;
+    a.nr_channels = plan->nr_channels;
+    a.nr_items = int64_t(plan->items.size());
+    a.items = dc->items;
+    a.order = dc->order;
+    a.baselines = dc->baselines;
+    a.frequencies = dc->frequencies;
+    a.uvw = d_uvw;
+    a.aterms = static_cast<const float2 *>(d_aterms);
+    a.taper = d_taper;
+    a.vis = static_cast<float2 *>(d_vis);
+    a.grid = static_cast<float2 *>(d_grid);
+    a.max_channels_in_item = plan->max_channels_in_item;
+    return a;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *idg_status_string(idg_status s) {
+    switch (s) {
+        case IDG_OK: return "IDG_OK";
+        case IDG_ERR_INVALID_ARG: return "IDG_ERR_INVALID_ARG";
+        case IDG_ERR_UNSUPPORTED: return "IDG_ERR_UNSUPPORTED";
+        case IDG_ERR_OUT_OF_MEMORY: return "IDG_ERR_OUT_OF_MEMORY";
+        case IDG_ERR_CUDA: return "IDG_ERR_CUDA";
+        case IDG_ERR_WORKSPACE_TOO_SMALL: return "IDG_ERR_WORKSPACE_TOO_SMALL";
+    }
+    return "IDG_ERR_UNKNOWN";
+}
+
+const char *idg_last_error(void) { return g_last_error.c_str(); }
+
+int64_t idg_launch_count(void) { return g_launches.load(); }
+
+idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, int32_t nr_baselines,
+                           int32_t nr_timesteps, int32_t nr_channels, const float *uvw,
+                           const double *frequencies, const idg_baseline *baselines,
+                           int32_t nr_aterm_slots, const int32_t *aterm_offsets, idg_plan **out) {
+    try {
+        if (!out) return fail(IDG_ERR_INVALID_ARG, "out is NULL");
+        *out = nullptr;
+        idg_status st = validate_params(params);
+        if (st != IDG_OK) return st;
+        if (nr_stations < 2 || nr_baselines < 0 || nr_timesteps < 1 || nr_channels < 1 ||
+            nr_aterm_slots < 1)
+            return fail(IDG_ERR_INVALID_ARG, "need nr_stations >= 2, nr_baselines >= 0, "
+                                             "nr_timesteps >= 1, nr_channels >= 1, nr_aterm_slots >= 1");
+        if ((nr_baselines > 0 && (!uvw || !baselines)) || !frequencies || !aterm_offsets)
+            return fail(IDG_ERR_INVALID_ARG, "NULL host array");
+        for (int32_t c = 0; c < nr_channels; ++c)
+            if (!(frequencies[c] > 0.0) || !std::isfinite(frequencies[c]))
+                return fail(IDG_ERR_INVALID_ARG, "frequencies must be positive and finite");
+        if (aterm_offsets[0] != 0 || aterm_offsets[nr_aterm_slots] != nr_timesteps)
+            return fail(IDG_ERR_INVALID_ARG, "aterm_offsets must start at 0 and end at nr_timesteps");
+        for (int32_t s = 0; s < nr_aterm_slots; ++s)
+            if (aterm_offsets[s + 1] <= aterm_offsets[s])
+                return fail(IDG_ERR_INVALID_ARG, "aterm_offsets must be strictly increasing");
+        for (int32_t b = 0; b < nr_baselines; ++b)
+            if (baselines[b].station1 < 0 || baselines[b].station1 >= baselines[b].station2 ||
+                baselines[b].station2 >= nr_stations)
+                return fail(IDG_ERR_INVALID_ARG, "baseline " + std::to_string(b) +
+                                                     ": need 0 <= station1 < station2 < nr_stations");
+
+        auto plan = std::make_unique<idg_plan>();
+        plan->params = *params;
+        plan->nr_stations = nr_stations;
+        plan->nr_baselines = nr_baselines;
+        plan->nr_timesteps = nr_timesteps;
+        plan->nr_channels = nr_channels;
+        plan->nr_aterm_slots = nr_aterm_slots;
+        plan->frequencies.assign(frequencies, frequencies + nr_channels);
+        plan->baselines.resize(size_t(nr_baselines) * 2);
+        for (int32_t b = 0; b < nr_baselines; ++b) {
+            plan->baselines[2 * b] = baselines[b].station1;
+            plan->baselines[2 * b + 1] = baselines[b].station2;
+        }
+        idg::PlanResult res;
+        std::string err;
+        st = idg::build_plan(*params, nr_stations, nr_baselines, nr_timesteps, nr_channels, uvw,
+                             frequencies, baselines, nr_aterm_slots, aterm_offsets, plan->items, res, err);
+        if (st != IDG_OK) return fail(st, err);
+        if (plan->items.size() > size_t(0x7fffffff))
+            return fail(IDG_ERR_UNSUPPORTED, "more than 2^31-1 work items");
+        plan->nr_vis_assigned = res.nr_vis_assigned;
+        plan->nr_vis_dropped = res.nr_vis_dropped;
+        const int64_t npix = int64_t(params->subgrid_size) * params->subgrid_size;
+        int g = 0;
+        for (const auto &it : plan->items) {
+            const int nc = it.channel_end - it.channel_begin;
+            plan->nr_pairs += npix * it.nr_timesteps * nc;
+            plan->max_channels_in_item = std::max(plan->max_channels_in_item, nc);
+            g = std::gcd(g, nc);
+        }
+        plan->degridder_v = idg::degridder_channels_per_thread(g == 0 ? 1 : g);
+        plan->order.resize(plan->items.size());
+        std::iota(plan->order.begin(), plan->order.end(), 0);
+        std::stable_sort(plan->order.begin(), plan->order.end(), [&](int32_t a, int32_t b) {
+            const auto &ia = plan->items[a], &ib = plan->items[b];
+            return int64_t(ia.nr_timesteps) * (ia.channel_end - ia.channel_begin) >
+                   int64_t(ib.nr_timesteps) * (ib.channel_end - ib.channel_begin);
+        });
+        *out = plan.release();
+        return IDG_OK;
+    } catch (const std::bad_alloc &) {
+        return fail(IDG_ERR_OUT_OF_MEMORY, "host allocation failed in idg_plan_create");
+    } catch (const std::exception &e) {
+        return fail(IDG_ERR_INVALID_ARG, e.what());
+    }
+}
+
+idg_status idg_plan_destroy(idg_plan *plan) {
+    delete plan;
+    return IDG_OK;
+}
+
+idg_status idg_plan_nr_subgrids(const idg_plan *plan, int64_t *n) {
+    if (!plan || !n) return fail(IDG_ERR_INVALID_ARG, "NULL argument");
+    *n = int64_t(plan->items.size());
+    return IDG_OK;
+}
+
+idg_status idg_plan_metadata(const idg_plan *plan, idg_metadata *dst, int64_t n) {
+    if (!plan || (!dst && n > 0) || n < 0) return fail(IDG_ERR_INVALID_ARG, "bad argument");
+    const int64_t k = std::min<int64_t>(n, int64_t(plan->items.size()));
+    if (k > 0) std::memcpy(dst, plan->items.data(), size_t(k) * sizeof(idg_metadata));
+    return IDG_OK;
+}
+
+idg_status idg_plan_stats(const idg_plan *plan, int64_t *assigned, int64_t *dropped, int64_t *pairs) {
+    if (!plan) return fail(IDG_ERR_INVALID_ARG, "plan is NULL");
+    if (assigned) *assigned = plan->nr_vis_assigned;
+    if (dropped) *dropped = plan->nr_vis_dropped;
+    if (pairs) *pairs = plan->nr_pairs;
+    return IDG_OK;
+}
+
+idg_status idg_workspace_size(const idg_plan *plan, size_t *bytes) {
+    if (!plan || !bytes) return fail(IDG_ERR_INVALID_ARG, "NULL argument");
+    *bytes = 0;  // gridder/degridder are fused with FFT + adder/splitter: no subgrid round trip
+    return IDG_OK;
+}
+
+idg_status idg_grid(const idg_plan *plan, const void *d_vis, const float *d_uvw, const void *d_aterms,
+                    const float *d_taper, void *d_grid, void *d_workspace, size_t workspace_bytes,
+                    idg_stream stream) {
+    (void)d_workspace;
+    (void)workspace_bytes;
+    try {
+        idg_status st = validate_call(plan, d_vis, d_uvw, d_aterms, d_taper, d_grid);
+        if (st != IDG_OK || plan->items.empty()) return st;
+        const DeviceCopy *dc = nullptr;
+        if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper, const_cast<void *>(d_vis), d_grid);
+        cudaError_t e = idg::launch_gridder(a, reinterpret_cast<cudaStream_t>(stream));
+        if (e != cudaSuccess) return cuda_fail(e, "gridder launch");
+        return IDG_OK;
+    } catch (const std::exception &ex) {
+        return fail(IDG_ERR_INVALID_ARG, ex.what());
+    }
+}
+
+idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_uvw, const void *d_aterms,
+                      const float *d_taper, void *d_vis, void *d_workspace, size_t workspace_bytes,
+                      idg_stream stream) {
+    (void)d_workspace;
+    (void)workspace_bytes;
+    try {
+        if (!plan) return fail(IDG_ERR_INVALID_ARG, "plan is NULL");
+        const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+        if (plan->nr_vis_dropped > 0 || plan->items.empty()) {
+            // dropped visibilities are defined as 0 (R-12, R-13); items overwrite the rest
+            if (!d_vis) return fail(IDG_ERR_INVALID_ARG, "d_vis is NULL");
+            const size_t bytes = size_t(plan->nr_baselines) * plan->nr_timesteps * plan->nr_channels * 32;
+            cudaError_t e = cudaMemsetAsync(d_vis, 0, bytes, s);
+            if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(vis)");
+        }
+        idg_status st = validate_call(plan, d_vis, d_uvw, d_aterms, d_taper, d_grid);
+        if (st != IDG_OK || plan->items.empty()) return st;
+        const DeviceCopy *dc = nullptr;
+        if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper, d_vis, const_cast<void *>(d_grid));
+        cudaError_t e = idg::launch_degridder_v(a, plan->degridder_v, s);
+        if (e != cudaSuccess) return cuda_fail(e, "degridder launch");
+        return IDG_OK;
+    } catch (const std::exception &ex) {
+        return fail(IDG_ERR_INVALID_ARG, ex.what());
+    }
+}
+
+idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
+                             double *seconds) {
+    if (rho < 1 || rho > 64 || iterations < 1 || !ops_per_second)
+        return fail(IDG_ERR_INVALID_ARG, "rho in [1,64], iterations >= 1, ops_per_second != NULL");
+    const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    float *d_out = nullptr;
+    cudaError_t e = cudaMalloc(&d_out, sizeof(float) * 148 * 64 * 256);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(rho)");
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    int blocks = 0, threads = 0, units = 0;
+    // warm-up launch, then the timed one
+    e = idg::launch_rho_benchmark(rho, std::max(1, iterations / 8), d_out, s, &blocks, &threads, &units);
+    if (e == cudaSuccess) {
+        cudaEventRecord(e0, s);
+        e = idg::launch_rho_benchmark(rho, iterations, d_out, s, &blocks, &threads, &units);
+        cudaEventRecord(e1, s);
+    }
+    if (e == cudaSuccess) e = cudaEventSynchronize(e1);
+    float ms = 0.0f;
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, e0, e1);
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(d_out);
+    if (e != cudaSuccess) return cuda_fail(e, "rho benchmark");
+    const double sincos = double(blocks) * threads * units * double(iterations);
+    const double ops = sincos * (2.0 * rho + 2.0);  // rho FMAs (2 ops each) + sin + cos
+    *ops_per_second = ops / (double(ms) * 1e-3);
+    if (seconds) *seconds = double(ms) * 1e-3;
+    return IDG_OK;
+}
+
+idg_status idg_profiling_enable(int32_t enable) {
+    g_prof_enabled.store(enable != 0);
+    return IDG_OK;
+}
+
+static void drain_profiling_locked() {
+    for (auto &r : g_prof_pending) {
+        cudaEventSynchronize(r.e1);
+        float ms = 0.0f;
+        cudaEventElapsedTime(&ms, r.e0, r.e1);
+        auto &t = g_prof_totals[r.name];
+        t.first += 1;
+        t.second += ms;
+        cudaEventDestroy(r.e0);
+        cudaEventDestroy(r.e1);
+    }
+    g_prof_pending.clear();
+}
+
+idg_status idg_profiling_reset(void) {
+    std::lock_guard<std::mutex> lock(g_prof_mu);
+    drain_profiling_locked();
+    g_prof_totals.clear();
+    return IDG_OK;
+}
+
+idg_status idg_profiling_read(idg_kernel_time *dst, int32_t capacity, int32_t *n) {
+    if (!n || (capacity > 0 && !dst)) return fail(IDG_ERR_INVALID_ARG, "bad argument");
+    std::lock_guard<std::mutex> lock(g_prof_mu);
+    drain_profiling_locked();
+    int32_t k = 0;
+    for (auto &kv : g_prof_totals) {
+        if (k < capacity) {
+            std::memset(dst[k].name, 0, sizeof(dst[k].name));
+            std::strncpy(dst[k].name, kv.first.c_str(), sizeof(dst[k].name) - 1);
+            dst[k].launches = kv.second.first;
+            dst[k].total_ms = kv.second.second;
+        }
+        ++k;
+    }
+    *n = k;
+    return IDG_OK;
+}
+
+}  // extern "C"

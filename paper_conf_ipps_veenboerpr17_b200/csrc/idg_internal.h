@@ -1,0 +1,66 @@
+// idg_internal.h -- structures shared by the host API (idg_api.cpp, idg_plan.cpp) and the sm_100a
+// kernels (idg_kernels.cu).  Not part of the public ABI (see include/idg.h).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+#include <cuda_runtime.h>
+
+#include "idg.h"
+
+namespace idg {
+
+constexpr double kSpeedOfLight = 299792458.0;  // m/s; u_lambda = u nu / c
+
+// Host-side result of the plan builder.
+struct PlanResult {
+    int64_t nr_vis_assigned = 0;
+    int64_t nr_vis_dropped = 0;
+};
+
+// Builds the work items; `items` is cleared and filled in plan order.  Returns IDG_OK or an error
+// (with a message in `err`).
+idg_status build_plan(const idg_plan_params &p, int32_t nr_stations, int32_t nbl, int32_t T,
+                      int32_t C, const float *uvw, const double *freqs,
+                      const idg_baseline *baselines, int32_t nslots, const int32_t *aterm_offsets,
+                      std::vector<idg_metadata> &items, PlanResult &res, std::string &err);
+
+// Arguments of the fused gridder / degridder launches (device pointers).
+struct KernelArgs {
+    int32_t subgrid_size;        // N~
+    int32_t grid_size;           // N
+    float cell_l;                // L / N~   (direction-cosine step of a subgrid pixel)
+    double inv_image_size;       // du = 1/L (wavelengths per grid cell)
+    double w_offset;             // w0
+    int32_t nr_stations, nr_baselines, nr_timesteps, nr_channels;
+    int64_t nr_items;
+    const idg_metadata *items;   // [nr_items]
+    const int32_t *order;        // [nr_items] launch order (largest work first)
+    const int32_t *baselines;    // [nbl][2]
+    const double *frequencies;   // [C] Hz
+    const float *uvw;            // [nbl][T][3]
+    const float2 *aterms;        // [slots][S][N~][N~][4]
+    const float *taper;          // [N~][N~]
+    float2 *vis;                 // [nbl][T][C][4]  (const for gridding)
+    float2 *grid;                // [4][N][N]       (const for degridding)
+    int32_t max_channels_in_item;
+};
+
+cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s);
+// V = channels per degridder thread; every item's channel count must be a multiple of V.
+int degridder_channels_per_thread(int channel_gcd);
+cudaError_t launch_degridder_v(const KernelArgs &a, int V, cudaStream_t s);
+cudaError_t launch_rho_benchmark(int rho, int iterations, float *d_out, cudaStream_t s,
+                                 int *blocks, int *threads, int *units_per_thread);
+
+// Kernel-launch bookkeeping (profiling + launch counter), idg_api.cpp.
+struct LaunchScope {
+    LaunchScope(const char *name, cudaStream_t s);
+    ~LaunchScope();
+    const char *name;
+    cudaStream_t stream;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+};
+
+}  // namespace idg

@@ -1,0 +1,145 @@
+"""GPU parity: the sm_100a path (through the C ABI) against the fp64 oracle, element by element.
+
+Bar (BASELINE.json north_star): relative RMS error ||x - x_oracle||_2 / ||x_oracle||_2 <= 1e-4 on grids
+(all cells x pols) and on visibilities (all visibilities x pols); the plan is bit-exact (test_abi_plan).
+Sizes span several work items, ragged channel blocks, every subgrid size (16/24/32) and both grid sizes
+of the configs; full-size configs are checked on sampled work items (the oracle computes them one by
+one) and through the adjoint identity, which holds at any size.
+"""
+import numpy as np
+import pytest
+
+import idgsynth
+import oracle
+
+torch = pytest.importorskip("torch")
+import paper_conf_ipps_veenboerpr17_b200 as idg
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-4
+
+
+def rel_rms(x, ref):
+    x = np.asarray(x).astype(np.complex128).reshape(-1)
+    ref = np.asarray(ref).astype(np.complex128).reshape(-1)
+    return float(np.linalg.norm(x - ref) / np.linalg.norm(ref))
+
+
+def _inputs(obs, aterm_kind=None, taper_kind="spheroidal"):
+    vis = idgsynth.make_visibilities(obs)
+    aterms = idgsynth.make_aterms(obs, aterm_kind)
+    taper = idgsynth.make_taper(obs.subgrid_size, taper_kind)
+    return vis, aterms, taper
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def gpu_grid(obs, vis, aterms, taper, plan=None):
+    plan = plan or idg.Plan.from_observation(obs)
+    N = obs.grid_size
+    g = torch.zeros((4, N, N), dtype=torch.complex64, device="cuda")
+    idg.grid(plan, _dev(vis), _dev(obs.uvw), _dev(aterms), _dev(taper), g)
+    torch.cuda.synchronize()
+    return g
+
+
+def gpu_degrid(obs, grid_np_or_t, aterms, taper, plan=None):
+    plan = plan or idg.Plan.from_observation(obs)
+    g = grid_np_or_t if isinstance(grid_np_or_t, torch.Tensor) else _dev(grid_np_or_t)
+    v = torch.full((obs.nr_baselines, obs.nr_timesteps, obs.nr_channels, 4), complex(7, 7),
+                   dtype=torch.complex64, device="cuda")
+    idg.degrid(plan, g, _dev(obs.uvw), _dev(aterms), _dev(taper), v)
+    torch.cuda.synchronize()
+    return v
+
+
+CASES = [
+    ("tiny", {}, "identity", "ones"),
+    ("tiny", {}, "identity", "spheroidal"),
+    ("small_dde", {}, None, "spheroidal"),
+    ("small_dde", dict(C=7, C_block=3), None, "spheroidal"),          # ragged channel blocks
+    ("small_dde", dict(C=12), None, "spheroidal"),                   # 12 channels: V=4 degridder
+    ("lofar", dict(T=640, nr_stations=5), None, "spheroidal"),       # N~=24, N=2048, 16 ch
+    ("lofar_dde", dict(T=512, nr_stations=5), None, "spheroidal"),   # + random A-terms, w0
+    ("ska", dict(T=384, nr_stations=4), None, "spheroidal"),         # N~=32, N=8192, 32 ch
+]
+
+
+@pytest.mark.parametrize("name,kw,aterm,taper", CASES)
+def test_grid_matches_oracle(name, kw, aterm, taper):
+    obs = idgsynth.make_observation(name, **kw)
+    vis, aterms, tap = _inputs(obs, aterm, taper)
+    items, _ = oracle.plan(obs)
+    ref = oracle.grid(obs, items, vis, aterms, tap)
+    got = gpu_grid(obs, vis, aterms, tap).cpu().numpy()
+    err = rel_rms(got, ref)
+    print(f"grid {name} {kw}: rel rms {err:.3e}")
+    assert err <= TOL, err
+
+
+@pytest.mark.parametrize("name,kw,aterm,taper", CASES)
+def test_degrid_matches_oracle(name, kw, aterm, taper):
+    obs = idgsynth.make_observation(name, **kw)
+    _, aterms, tap = _inputs(obs, aterm, taper)
+    G = idgsynth.make_grid(obs)
+    items, dropped = oracle.plan(obs)
+    ref = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, G, aterms, tap))
+    got = gpu_degrid(obs, G, aterms, tap).cpu().numpy()
+    err = rel_rms(got, ref)
+    print(f"degrid {name} {kw}: rel rms {err:.3e}")
+    assert err <= TOL, err
+
+
+def test_grid_accumulates_and_degrid_zeroes_dropped():
+    import dataclasses
+    obs = idgsynth.make_observation("small_dde")
+    obs = dataclasses.replace(obs, image_size=obs.image_size * 6)     # long baselines fall off the grid
+    vis, aterms, tap = _inputs(obs)
+    items, dropped = oracle.plan(obs)
+    assert dropped > 0
+    plan = idg.Plan.from_observation(obs)
+    g = gpu_grid(obs, vis, aterms, tap, plan)
+    idg.grid(plan, _dev(vis), _dev(obs.uvw), _dev(aterms), _dev(tap), g)    # second call accumulates
+    ref = 2 * oracle.grid(obs, items, vis, aterms, tap)
+    assert rel_rms(g.cpu().numpy(), ref) <= TOL
+    G = idgsynth.make_grid(obs)
+    got = gpu_degrid(obs, G, aterms, tap, plan).cpu().numpy()
+    ref = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, G, aterms, tap))
+    assert rel_rms(got, ref) <= TOL
+    covered = oracle.scatter_visibilities(obs, items, np.ones(int(np.sum(
+        items["nr_timesteps"] * (items["channel_end"] - items["channel_begin"]))) * 4))
+    assert np.all(got[covered == 0] == 0)                              # dropped -> exactly 0
+
+
+def _inner_t(a, b):
+    return torch.vdot(a.reshape(-1).to(torch.complex128), b.reshape(-1).to(torch.complex128)).item()
+
+
+@pytest.mark.parametrize("name", ["lofar_dde", "lofar"])
+def test_full_size_adjoint_and_sampled_items(name):
+    """Full LOFAR-shaped set in the bench launch configuration: <degrid(G),V> = <G,grid(V)> on the GPU,
+    and degridded visibilities of sampled work items against the oracle computing just those items."""
+    obs = idgsynth.make_observation(name)
+    aterms = idgsynth.make_aterms(obs)
+    tap = idgsynth.make_taper(obs.subgrid_size)
+    plan = idg.Plan.from_observation(obs)
+    uvw, at, tp = _dev(obs.uvw), _dev(aterms), _dev(tap)
+    V = idgsynth.torch_visibilities(obs, "cuda")
+    G = idgsynth.torch_grid(obs, "cuda")
+    gV = torch.zeros_like(G)
+    idg.grid(plan, V, uvw, at, tp, gV)
+    DG = torch.empty_like(V)
+    idg.degrid(plan, G, uvw, at, tp, DG)
+    torch.cuda.synchronize()
+    lhs, rhs = _inner_t(DG, V), _inner_t(G, gV)
+    assert abs(lhs - rhs) / abs(lhs) < 1e-4, (lhs, rhs)
+    # sampled items through the oracle
+    items, _ = oracle.plan(obs)
+    rng = np.random.default_rng(0)
+    sel = items[np.sort(rng.choice(len(items), 24, replace=False))]
+    Gh = G.cpu().numpy()
+    ref = oracle.degrid(obs, sel, Gh, aterms, tap)
+    got = oracle.gather_visibilities(obs, sel, DG.cpu().numpy())
+    assert rel_rms(got, ref) <= TOL
