@@ -142,10 +142,14 @@ def earth_rotation_uvw(xyz, baselines, nr_timesteps, dt, dec):
     return np.stack([u, v, w], axis=2).astype(np.float32)
 
 
+MAX_IMAGE_SIZE = 0.3
+
+
 def image_size_for(uvw, frequencies, grid_size, subgrid_size):
-    """L = (N/2 - N~) / max|u_lambda, v_lambda| so that no subgrid falls off the grid."""
+    """L = (N/2 - N~) / max|u_lambda, v_lambda| so that no subgrid falls off the grid,
+    capped at 0.3 (a ~17 degree field) so that small station subsets still image a physical sky."""
     umax = float(np.max(np.abs(uvw[:, :, :2]).astype(np.float64))) * float(np.max(frequencies)) / SPEED_OF_LIGHT
-    return (grid_size / 2 - subgrid_size) / umax
+    return min(MAX_IMAGE_SIZE, (grid_size / 2 - subgrid_size) / umax)
 
 
 # ----------------------------------------------------------------------------------------------

@@ -49,7 +49,7 @@ typedef struct {
 typedef struct {
     int32_t subgrid_size;              /* N~: 16, 24 or 32 ("as small as 24x24")              */
     int32_t grid_size;                 /* N: even, >= 2 N~ (2048)                            */
-    double image_size;                 /* L (direction cosines); grid cell du = 1/L wavelengths     */
+    double image_size;                 /* L in (0, sqrt 2) (direction cosines); cell du = 1/L       */
     int32_t kernel_size;               /* K: support reserved around the footprint (Fig. 5; R-8)    */
     int32_t max_timesteps_per_subgrid; /* T~max >= 1 (R-14)                                   */
     int32_t max_channels_per_subgrid;  /* C~: channel block size; 0 = all channels (R-9)     */
@@ -136,7 +136,7 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
  * idg_rho_benchmark -- the paper's FMA:sincos throughput benchmark (Fig. 12) on the
  * current device: every sincos evaluation is followed by rho-1 FMAs plus the one FMA that forms its
  * argument (rho FMAs per sincos).  ops = 2 per FMA + 1 per sin + 1 per cos (op definition).
- *   rho in [1, 64];  iterations >= 1 (work per thread);  ops_per_second receives the measured
+ *   rho in {1,2,3,4,6,8,12,16,17,20,24,32,48,64};  iterations >= 1 (work per thread);  ops_per_second receives the measured
  *   throughput (synchronous: the call waits for the kernel; timed with CUDA events on `stream`).
  */
 idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream,
@@ -156,6 +156,11 @@ typedef struct {
 idg_status idg_profiling_enable(int32_t enable);
 idg_status idg_profiling_reset(void);
 idg_status idg_profiling_read(idg_kernel_time *dst, int32_t capacity, int32_t *n);
+
+/* Diagnostics: newline-separated names of the compiled launch-shape variants of the gridder
+ * (which = 0) or degridder (which = 1).  Setting the environment variable IDG_GRIDDER_VARIANT /
+ * IDG_DEGRIDDER_VARIANT to one of these names before a call overrides the default (tuning only). */
+const char *idg_kernel_variants(int32_t which);
 
 /* Number of kernel launches issued by this library in the calling process so far. */
 int64_t idg_launch_count(void);

@@ -151,8 +151,9 @@ idg_status validate_params(const idg_plan_params *p) {
                                              std::to_string(p->subgrid_size) + ")");
     if (p->grid_size < 2 * p->subgrid_size || p->grid_size % 2 != 0 || p->grid_size > (1 << 16))
         return fail(IDG_ERR_INVALID_ARG, "grid_size must be even, >= 2*subgrid_size and <= 65536");
-    if (!(p->image_size > 0.0) || !std::isfinite(p->image_size) || p->image_size >= 2.0)
-        return fail(IDG_ERR_INVALID_ARG, "image_size must be in (0, 2)");
+    // every subgrid pixel must be a direction on the sky: l^2 + m^2 < 1 at the corner (-L/2, -L/2)
+    if (!(p->image_size > 0.0) || !std::isfinite(p->image_size) || p->image_size >= 1.4142135)
+        return fail(IDG_ERR_INVALID_ARG, "image_size must be in (0, sqrt(2))");
     if (p->kernel_size < 0 || p->kernel_size >= p->subgrid_size)
         return fail(IDG_ERR_INVALID_ARG, "kernel_size must be in [0, subgrid_size)");
     if (p->max_timesteps_per_subgrid < 1)
@@ -217,6 +218,8 @@ const char *idg_status_string(idg_status s) {
 const char *idg_last_error(void) { return g_last_error.c_str(); }
 
 int64_t idg_launch_count(void) { return g_launches.load(); }
+
+const char *idg_kernel_variants(int32_t which) { return idg::variant_names(which == 0 ? 0 : 1); }
 
 idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, int32_t nr_baselines,
                            int32_t nr_timesteps, int32_t nr_channels, const float *uvw,
@@ -375,8 +378,11 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
 
 idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
                              double *seconds) {
-    if (rho < 1 || rho > 64 || iterations < 1 || !ops_per_second)
-        return fail(IDG_ERR_INVALID_ARG, "rho in [1,64], iterations >= 1, ops_per_second != NULL");
+    static const int kSupported[] = {1, 2, 3, 4, 6, 8, 12, 16, 17, 20, 24, 32, 48, 64};
+    if (std::find(std::begin(kSupported), std::end(kSupported), rho) == std::end(kSupported) ||
+        iterations < 1 || !ops_per_second)
+        return fail(IDG_ERR_INVALID_ARG,
+                    "rho in {1,2,3,4,6,8,12,16,17,20,24,32,48,64}, iterations >= 1, ops_per_second != NULL");
     const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
     float *d_out = nullptr;
     cudaError_t e = cudaMalloc(&d_out, sizeof(float) * 148 * 64 * 256);

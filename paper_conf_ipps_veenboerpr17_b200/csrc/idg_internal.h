@@ -51,6 +51,7 @@ cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s);
 // V = channels per degridder thread; every item's channel count must be a multiple of V.
 int degridder_channels_per_thread(int channel_gcd);
 cudaError_t launch_degridder_v(const KernelArgs &a, int V, cudaStream_t s);
+const char *variant_names(int which);
 cudaError_t launch_rho_benchmark(int rho, int iterations, float *d_out, cudaStream_t s,
                                  int *blocks, int *threads, int *units_per_thread);
 

@@ -23,6 +23,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <cstring>
+#include <string>
 
 #include "idg_internal.h"
 
@@ -129,8 +132,8 @@ inline size_t gridder_smem_bytes(int NS, int max_channels) {
     return std::max(main_loop, epi) + 16;
 }
 
-template <int NS, int P>
-__global__ void __launch_bounds__(NS *NS / P) gridder_kernel(const KernelArgs a) {
+template <int NS, int P, int MINB>
+__global__ void __launch_bounds__(NS *NS / P, MINB) gridder_kernel(const KernelArgs a) {
     constexpr int NT = NS * NS / P;
     constexpr int NPIX = NS * NS;
     constexpr int h = NS / 2;
@@ -316,8 +319,6 @@ __global__ void __launch_bounds__(NS *NS / P) gridder_kernel(const KernelArgs a)
 // are read as warp broadcasts (the thread's "first mapping" = visibilities, the
 // "second mapping" = pixels in the prologue).
 // ------------------------------------------------------------------------------------------------
-constexpr int kDegridderThreads = 256;
-
 inline size_t degridder_smem_bytes(int NS, int max_channels) {
     const size_t npix = size_t(NS) * NS;
     const size_t region_a = std::max(npix * 48, npix * 4 * sizeof(float2));  // pixels | split sub
@@ -325,9 +326,8 @@ inline size_t degridder_smem_bytes(int NS, int max_channels) {
     return region_a + region_b + size_t(max_channels) * 4 + 16;
 }
 
-template <int NS, int V>
-__global__ void __launch_bounds__(kDegridderThreads) degridder_kernel(const KernelArgs a) {
-    constexpr int NT = kDegridderThreads;
+template <int NS, int V, int NT, int MINB>
+__global__ void __launch_bounds__(NT, MINB) degridder_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int h = NS / 2;
     extern __shared__ __align__(16) unsigned char smem[];
@@ -478,50 +478,81 @@ __global__ void __launch_bounds__(kDegridderThreads) degridder_kernel(const Kern
     }
 }
 
-template <int NS, int P>
+template <typename K>
+cudaError_t prepare(K kernel, size_t smem) {
+    cudaError_t err = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    if (err != cudaSuccess) return err;
+    return cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                int(cudaSharedmemCarveoutMaxShared));
+}
+
+template <int NS, int P, int MINB>
 cudaError_t launch_gridder_t(const KernelArgs &a, cudaStream_t st) {
     constexpr int NT = NS * NS / P;
     static_assert(NS * NS % (P * 32) == 0, "pixels per thread must give whole warps");
     const size_t smem = gridder_smem_bytes(NS, a.max_channels_in_item);
-    cudaError_t err = cudaFuncSetAttribute(gridder_kernel<NS, P>,
-                                           cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    cudaError_t err = prepare(gridder_kernel<NS, P, MINB>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("gridder", st);
-    gridder_kernel<NS, P><<<unsigned(a.nr_items), NT, smem, st>>>(a);
+    gridder_kernel<NS, P, MINB><<<unsigned(a.nr_items), NT, smem, st>>>(a);
     return cudaGetLastError();
 }
 
-template <int NS, int V>
+template <int NS, int V, int NT, int MINB>
 cudaError_t launch_degridder_t(const KernelArgs &a, cudaStream_t st) {
     const size_t smem = degridder_smem_bytes(NS, a.max_channels_in_item);
-    cudaError_t err = cudaFuncSetAttribute(degridder_kernel<NS, V>,
-                                           cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    cudaError_t err = prepare(degridder_kernel<NS, V, NT, MINB>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("degridder", st);
-    degridder_kernel<NS, V><<<unsigned(a.nr_items), kDegridderThreads, smem, st>>>(a);
+    degridder_kernel<NS, V, NT, MINB><<<unsigned(a.nr_items), NT, smem, st>>>(a);
     return cudaGetLastError();
 }
 
-template <int NS>
-cudaError_t launch_degridder_ns(const KernelArgs &a, int V, cudaStream_t st) {
-    switch (V) {
-        case 8: return launch_degridder_t<NS, 8>(a, st);
-        case 4: return launch_degridder_t<NS, 4>(a, st);
-        case 2: return launch_degridder_t<NS, 2>(a, st);
-        default: return launch_degridder_t<NS, 1>(a, st);
+using Launcher = cudaError_t (*)(const KernelArgs &, cudaStream_t);
+struct Variant {
+    int ns, v;            // subgrid size; pixels (gridder) or channels (degridder) per thread
+    const char *name;
+    Launcher fn;
+};
+
+// Launch-shape variants (tuned on B200 with scripts/tune.py; the first entry per (NS, V) is the default).
+#define GV(NS, P, MB) {NS, 0, "gridder<" #NS ",P" #P ",minB" #MB ">", launch_gridder_t<NS, P, MB>}
+const Variant kGridderVariants[] = {
+    GV(24, 6, 4), GV(24, 6, 5), GV(24, 6, 6), GV(24, 3, 3), GV(24, 3, 4), GV(24, 2, 4), GV(24, 9, 3),
+    GV(32, 8, 3), GV(32, 8, 4), GV(32, 4, 2), GV(32, 4, 3), GV(32, 16, 4),
+    GV(16, 4, 4), GV(16, 4, 6), GV(16, 2, 4), GV(16, 8, 6),
+};
+#undef GV
+#define DV(NS, V, NT, MB) {NS, V, "degridder<" #NS ",V" #V ",T" #NT ",minB" #MB ">", launch_degridder_t<NS, V, NT, MB>}
+#define DV_ALL(NS) DV(NS, 8, 128, 3), DV(NS, 8, 128, 4), DV(NS, 8, 256, 1), DV(NS, 8, 256, 2), \
+    DV(NS, 8, 64, 6), DV(NS, 8, 64, 8), DV(NS, 4, 128, 4), DV(NS, 4, 256, 3), DV(NS, 4, 128, 6), \
+    DV(NS, 2, 128, 6), DV(NS, 1, 128, 6)
+const Variant kDegridderVariants[] = {DV_ALL(24), DV_ALL(32), DV_ALL(16)};
+#undef DV_ALL
+#undef DV
+
+// Variant choice: default = first match; env IDG_GRIDDER_VARIANT / IDG_DEGRIDDER_VARIANT = name
+// overrides (tuning only).
+template <size_t K>
+const Variant *pick(const Variant (&table)[K], int ns, int v, const char *env) {
+    const char *want = std::getenv(env);
+    const Variant *first = nullptr;
+    for (const Variant &var : table) {
+        if (var.ns != ns) continue;
+        // an override may use fewer channels per thread than the default, as long as it divides it
+        const bool valid = (v == 0) ? var.v == 0 : (var.v > 0 && v % var.v == 0);
+        if (valid && want && std::strcmp(want, var.name) == 0) return &var;
+        if (!first && var.v == v) first = &var;
     }
+    return first;
 }
 
 }  // namespace
 
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
-    switch (a.subgrid_size) {
-        case 16: return launch_gridder_t<16, 4>(a, s);
-        case 24: return launch_gridder_t<24, 6>(a, s);
-        case 32: return launch_gridder_t<32, 8>(a, s);
-        default: return cudaErrorInvalidValue;
-    }
+    const Variant *var = pick(kGridderVariants, a.subgrid_size, 0, "IDG_GRIDDER_VARIANT");
+    return var ? var->fn(a, s) : cudaErrorInvalidValue;
 }
 
 // The channel count of every item must be a multiple of V (the host picks V from the plan).
@@ -534,12 +565,17 @@ int degridder_channels_per_thread(int channel_gcd) {
 
 cudaError_t launch_degridder_v(const KernelArgs &a, int V, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
-    switch (a.subgrid_size) {
-        case 16: return launch_degridder_ns<16>(a, V, s);
-        case 24: return launch_degridder_ns<24>(a, V, s);
-        case 32: return launch_degridder_ns<32>(a, V, s);
-        default: return cudaErrorInvalidValue;
+    const Variant *var = pick(kDegridderVariants, a.subgrid_size, V, "IDG_DEGRIDDER_VARIANT");
+    return var ? var->fn(a, s) : cudaErrorInvalidValue;
+}
+
+const char *variant_names(int which) {
+    static std::string g, d;
+    if (g.empty()) {
+        for (const Variant &v : kGridderVariants) g += std::string(v.name) + "\n";
+        for (const Variant &v : kDegridderVariants) d += std::string(v.name) + "\n";
     }
+    return which == 0 ? g.c_str() : d.c_str();
 }
 
 }  // namespace idg

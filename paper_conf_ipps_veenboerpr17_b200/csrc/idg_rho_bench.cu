@@ -14,44 +14,45 @@
 namespace idg {
 namespace {
 
-constexpr int kRhoUnits = 8;
+constexpr int kRhoUnits = 4;
 constexpr int kRhoThreads = 256;
 
+// Per unit and iteration: the argument FMA consumes the previous sin and cos (so neither can be
+// dropped, at any rho), then rho-1 accumulate FMAs alternate over cos and sin into 8 accumulators.
 template <int RHO>
 __global__ void __launch_bounds__(kRhoThreads) rho_kernel(float *out, int iterations) {
     constexpr int U = kRhoUnits;
     const int tid = blockIdx.x * blockDim.x + threadIdx.x;
-    float B[U], Q[U], acc[U][8], coef[8];
+    float sn[U], cs[U], acc[U][8], coef[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) coef[j] = 0.25f + 0.01f * float((tid + j) & 7);
 #pragma unroll
     for (int k = 0; k < U; ++k) {
-        B[k] = 0.1f * float(k) + 1e-6f * float(tid & 1023);
-        Q[k] = 0.37f + 0.013f * float(k);
+        sn[k] = 0.1f * float(k) + 1e-6f * float(tid & 1023);
+        cs[k] = 0.37f + 0.013f * float(k);
 #pragma unroll
         for (int j = 0; j < 8; ++j) acc[k][j] = 0.0f;
     }
-    float x = 1e-3f * float(tid & 255);
+    const float x = 0.731f + 1e-7f * float(tid & 255);
 #pragma unroll 1
     for (int i = 0; i < iterations; ++i) {
-        x += 0.0009765625f;
 #pragma unroll
         for (int k = 0; k < U; ++k) {
-            const float ph = fmaf(x, Q[k], B[k]);  // FMA #1: the argument f().g()
-            float sn, cs;
-            __sincosf(ph, &sn, &cs);
+            const float ph = fmaf(x, cs[k], sn[k]);  // FMA #1: the argument f().g()
+            __sincosf(ph, &sn[k], &cs[k]);
 #pragma unroll
-            for (int j = 0; j < RHO - 1; ++j) {   // FMAs #2 .. #rho
-                const int a = j & 7;
-                acc[k][a] = fmaf(coef[(j >> 3) & 7], (j & 8) ? sn : cs, acc[k][a]);
+            for (int j = 0; j < RHO - 1; ++j) {       // FMAs #2 .. #rho
+                acc[k][j & 7] = fmaf(coef[(j >> 3) & 7], (j & 1) ? sn[k] : cs[k], acc[k][j & 7]);
             }
         }
     }
     float sum = 0.0f;
 #pragma unroll
-    for (int k = 0; k < U; ++k)
+    for (int k = 0; k < U; ++k) {
+        sum += sn[k] + cs[k];
 #pragma unroll
         for (int j = 0; j < 8; ++j) sum += acc[k][j];
+    }
     out[tid] = sum;
 }
 

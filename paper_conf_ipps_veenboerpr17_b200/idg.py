@@ -45,6 +45,7 @@ _lib = None
 EXPORTED = ["idg_plan_create", "idg_plan_destroy", "idg_plan_nr_subgrids", "idg_plan_metadata",
             "idg_plan_stats", "idg_workspace_size", "idg_grid", "idg_degrid", "idg_rho_benchmark",
             "idg_profiling_enable", "idg_profiling_reset", "idg_profiling_read", "idg_launch_count",
+            "idg_kernel_variants",
             "idg_status_string", "idg_last_error"]
 
 
@@ -72,11 +73,13 @@ def lib() -> ctypes.CDLL:
     L.idg_profiling_enable.argtypes = [i32]
     L.idg_profiling_read.argtypes = [ctypes.POINTER(KernelTime), i32, ctypes.POINTER(i32)]
     L.idg_launch_count.restype = i64
+    L.idg_kernel_variants.restype = ctypes.c_char_p
+    L.idg_kernel_variants.argtypes = [i32]
     L.idg_status_string.restype = ctypes.c_char_p
     L.idg_status_string.argtypes = [i32]
     L.idg_last_error.restype = ctypes.c_char_p
     for f in EXPORTED:
-        if f not in ("idg_launch_count", "idg_status_string", "idg_last_error"):
+        if f not in ("idg_launch_count", "idg_status_string", "idg_last_error", "idg_kernel_variants"):
             getattr(L, f).restype = i32
     _lib = L
     return L
@@ -238,6 +241,11 @@ def profiling_read() -> dict:
     _check(lib().idg_profiling_read(buf, 32, ctypes.byref(n)), "idg_profiling_read")
     return {buf[i].name.decode(): {"launches": int(buf[i].launches), "total_ms": float(buf[i].total_ms)}
             for i in range(min(n.value, 32))}
+
+
+def kernel_variants(which: str) -> list[str]:
+    """Compiled launch-shape variants of the 'gridder' or 'degridder' (see IDG_*_VARIANT)."""
+    return lib().idg_kernel_variants(0 if which == "gridder" else 1).decode().split()
 
 
 def launch_count() -> int:

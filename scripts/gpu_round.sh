@@ -17,7 +17,7 @@ if [ "${NCU:-1}" = "1" ]; then
   timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_$TAG.csv \
       python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1; echo "ncu launches rc=$?"
   for K in gridder degridder; do
-    timeout 900 ncu --set full --clock-control none --import-source on -k regex:${K}_kernel -s 1 -c 1 \
+    timeout 900 ncu --set full --clock-control none --import-source on -k regex:^${K}_kernel -s 1 -c 1 \
         -o $OUT/prof_${K}_$TAG -f python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > $OUT/ncu_${K}_$TAG.log 2>&1
     echo "ncu $K rc=$?"
   done
