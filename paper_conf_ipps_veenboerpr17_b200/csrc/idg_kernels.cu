@@ -519,12 +519,12 @@ struct Variant {
 #define GV(NS, P, MB) {NS, 0, "gridder<" #NS ",P" #P ",minB" #MB ">", launch_gridder_t<NS, P, MB>}
 const Variant kGridderVariants[] = {
     GV(24, 6, 4), GV(24, 6, 5), GV(24, 6, 6), GV(24, 3, 3), GV(24, 3, 4), GV(24, 2, 4), GV(24, 9, 3),
-    GV(32, 8, 3), GV(32, 8, 4), GV(32, 4, 2), GV(32, 4, 3), GV(32, 16, 4),
+    GV(32, 4, 2), GV(32, 8, 3), GV(32, 8, 4), GV(32, 4, 3), GV(32, 16, 4),
     GV(16, 4, 4), GV(16, 4, 6), GV(16, 2, 4), GV(16, 8, 6),
 };
 #undef GV
 #define DV(NS, V, NT, MB) {NS, V, "degridder<" #NS ",V" #V ",T" #NT ",minB" #MB ">", launch_degridder_t<NS, V, NT, MB>}
-#define DV_ALL(NS) DV(NS, 8, 128, 3), DV(NS, 8, 128, 4), DV(NS, 8, 256, 1), DV(NS, 8, 256, 2), \
+#define DV_ALL(NS) DV(NS, 8, 128, 4), DV(NS, 8, 128, 3), DV(NS, 8, 256, 1), DV(NS, 8, 256, 2), \
     DV(NS, 8, 64, 6), DV(NS, 8, 64, 8), DV(NS, 4, 128, 4), DV(NS, 4, 256, 3), DV(NS, 4, 128, 6), \
     DV(NS, 2, 128, 6), DV(NS, 1, 128, 6)
 const Variant kDegridderVariants[] = {DV_ALL(24), DV_ALL(32), DV_ALL(16)};
