@@ -105,13 +105,6 @@ def dist_env():
     return rank, world, local
 
 
-def shard_range(nbl: int, rank: int, world: int):
-    """Contiguous baseline shard of rank r (work per baseline = its visibilities x N~^2)."""
-    b0 = (nbl * rank) // world
-    b1 = (nbl * (rank + 1)) // world
-    return b0, b1
-
-
 def workload_description(name):
     obs_cfg = idgsynth.CONFIGS[name]
     return (f"{BASELINE['configs'][CONFIG_NAMES[name]]} | synthetic: {obs_cfg['nr_stations']} stations, "
@@ -199,7 +192,7 @@ def run_ours(args):
     import torch.distributed as dist
 
     import paper_conf_ipps_veenboerpr17_b200 as idg
-    from paper_conf_ipps_veenboerpr17_b200 import _build
+    from paper_conf_ipps_veenboerpr17_b200 import _build, parallel
     if not os.path.exists(_build.LIB):
         _build.build()
 
@@ -210,7 +203,7 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=dev)
 
     full = idgsynth.make_observation(args.config)
-    b0, b1 = shard_range(full.nr_baselines, rank, world)
+    b0, b1 = parallel.shard_range(full.nr_baselines, rank, world)
     obs = full.subset(nr_baselines=b1 - b0, baseline_begin=b0)
     t0 = time.perf_counter()
     plan = idg.Plan.from_observation(obs)
@@ -230,13 +223,12 @@ def run_ours(args):
     grid_d = torch.zeros((4, N, N), dtype=torch.complex64, device=dev)
     stream = torch.cuda.current_stream(dev)
 
+    sharded = parallel.ShardedIDG(plan)
+
     def step(vis_in, vis_out):
         grid_d.zero_()
-        idg.grid(plan, vis_in, uvw_d, at_d, tp_d, grid_d)
-        if world > 1:
-            dist.reduce(grid_d, dst=0)          # a5 across ranks: sum of the per-shard uv-grids
-            dist.broadcast(grid_d, src=0)       # the model grid for degridding (here: the gridded data)
-        idg.degrid(plan, grid_d, uvw_d, at_d, tp_d, vis_out)
+        sharded.grid(vis_in, uvw_d, at_d, tp_d, grid_d, dst=0)       # + NCCL reduce of the uv-grids
+        sharded.degrid(grid_d, uvw_d, at_d, tp_d, vis_out, src=0)    # NCCL broadcast of the model grid
 
     def barrier():
         if world > 1:
