@@ -62,7 +62,7 @@ struct idg_plan {
     std::vector<int32_t> order;      // launch order: largest T~ C~ first (tail balance)
     int64_t nr_vis_assigned = 0, nr_vis_dropped = 0, nr_pairs = 0;
     int32_t max_channels_in_item = 0;
-    int32_t degridder_v = 1;
+    int32_t channel_gcd = 1;
     mutable std::mutex mu;
     mutable std::map<int, DeviceCopy> device;
 
@@ -196,6 +196,7 @@ idg::KernelArgs make_args(const idg_plan *plan, const DeviceCopy *dc, const floa
     a.vis = static_cast<float2 *>(d_vis);
     a.grid = static_cast<float2 *>(d_grid);
     a.max_channels_in_item = plan->max_channels_in_item;
+    a.channel_gcd = plan->channel_gcd;
     return a;
 }
 
@@ -280,7 +281,7 @@ idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, i
             plan->max_channels_in_item = std::max(plan->max_channels_in_item, nc);
             g = std::gcd(g, nc);
         }
-        plan->degridder_v = idg::degridder_channels_per_thread(g == 0 ? 1 : g);
+        plan->channel_gcd = g == 0 ? 1 : g;
         plan->order.resize(plan->items.size());
         std::iota(plan->order.begin(), plan->order.end(), 0);
         std::stable_sort(plan->order.begin(), plan->order.end(), [&](int32_t a, int32_t b) {
@@ -368,7 +369,7 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
         const DeviceCopy *dc = nullptr;
         if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
         idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper, d_vis, const_cast<void *>(d_grid));
-        cudaError_t e = idg::launch_degridder_v(a, plan->degridder_v, s);
+        cudaError_t e = idg::launch_degridder(a, s);
         if (e != cudaSuccess) return cuda_fail(e, "degridder launch");
         return IDG_OK;
     } catch (const std::exception &ex) {

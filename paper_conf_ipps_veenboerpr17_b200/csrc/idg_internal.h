@@ -45,12 +45,24 @@ struct KernelArgs {
     float2 *vis;                 // [nbl][T][C][4]  (const for gridding)
     float2 *grid;                // [4][N][N]       (const for degridding)
     int32_t max_channels_in_item;
+    int32_t channel_gcd;         // gcd of all items' channel counts
 };
 
+using Launcher = cudaError_t (*)(const KernelArgs &, cudaStream_t);
+constexpr int kSimt = 0, kTensor = 1;
+struct Variant {
+    int ns;            // subgrid size
+    int v;             // channels per thread (SIMT degridder) / channel multiple (tensor gridder); 0 = any
+    int kind;          // kSimt | kTensor
+    const char *name;
+    Launcher fn;
+};
+// Tensor-core variants (idg_kernels_tc.cu); the first eligible one is the default.
+const Variant *tc_gridder_variants(int *n);
+const Variant *tc_degridder_variants(int *n);
+
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s);
-// V = channels per degridder thread; every item's channel count must be a multiple of V.
-int degridder_channels_per_thread(int channel_gcd);
-cudaError_t launch_degridder_v(const KernelArgs &a, int V, cudaStream_t s);
+cudaError_t launch_degridder(const KernelArgs &a, cudaStream_t s);
 const char *variant_names(int which);
 cudaError_t launch_rho_benchmark(int rho, int iterations, float *d_out, cudaStream_t s,
                                  int *blocks, int *threads, int *units_per_thread);

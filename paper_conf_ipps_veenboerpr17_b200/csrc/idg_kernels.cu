@@ -1,4 +1,5 @@
-// idg_kernels.cu -- sm_100a kernels of the IDG hot path (Veenboer, Petschow, Romein, IPDPS 2017).
+// idg_kernels.cu -- SIMT sm_100a kernels of the IDG hot path (Veenboer, Petschow, Romein, IPDPS 2017)
+// and the launch-variant dispatch (SIMT + tensor-core kernels of idg_kernels_tc.cu).
 //
 //   gridder_kernel    one CTA per work item: Alg. 1 (pixel = direct sum of phase-
 //                     shifted visibilities) -> A-term + taper (a3) -> centred subgrid DFT (a4)
@@ -27,96 +28,13 @@
 #include <cstring>
 #include <string>
 
+#include "idg_device.cuh"
 #include "idg_internal.h"
 
 namespace idg {
 namespace {
 
-constexpr double kTwoPi = 6.283185307179586476925286766559;
-
-__device__ __forceinline__ float2 cmul(float2 a, float2 b) {
-    return make_float2(a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x);
-}
-__device__ __forceinline__ float2 cmulc(float2 a, float2 b) {  // conj(a) * b
-    return make_float2(a.x * b.x + a.y * b.y, a.x * b.y - a.y * b.x);
-}
-__device__ __forceinline__ float2 cmul_conj_b(float2 a, float2 b) {  // a * conj(b)
-    return make_float2(a.x * b.x + a.y * b.y, a.y * b.x - a.x * b.y);
-}
-__device__ __forceinline__ float2 cadd(float2 a, float2 b) { return make_float2(a.x + b.x, a.y + b.y); }
-__device__ __forceinline__ float2 cscale(float2 a, float s) { return make_float2(a.x * s, a.y * s); }
-
-__device__ __forceinline__ float w_term_n(float l, float m) {
-    const float r2 = l * l + m * m;
-    return r2 / (1.0f + sqrtf(1.0f - r2));  // == 1 - sqrt(1 - r2)
-}
-
-// Streaming 16-byte load that does not allocate in L1 (visibilities are read once per item).
-__device__ __forceinline__ float4 ld_stream(const float4 *p) {
-    float4 v;
-    asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
-                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-                 : "l"(p));
-    return v;
-}
-
-// Vector fp32 atomic add of one complex value (sm_90+: red.global.add.v2.f32).
-__device__ __forceinline__ void red_add(float2 *addr, float2 v) {
-    asm volatile("red.global.add.v2.f32 [%0], {%1, %2};" ::"l"(addr), "f"(v.x), "f"(v.y)
-                 : "memory");
-}
-
-// Centred-DFT twiddle table tw[r] = exp(sign 2 pi i r / N~), r = 0..N~-1 (R-5).
-template <int NS>
-__device__ __forceinline__ void init_twiddles(float2 *tw, float sign) {
-    for (int r = threadIdx.x; r < NS; r += blockDim.x) {
-        float s, c;
-        sincospif(2.0f * float(r) / float(NS), &s, &c);
-        tw[r] = make_float2(c, sign * s);
-    }
-}
-
-// exponent index ((k - N~/2) (x - N~/2)) mod N~ at x = 0, and its increment per x
-template <int NS>
-__device__ __forceinline__ void dft_index(int k, int &idx0, int &step) {
-    constexpr int h = NS / 2;
-    int e = (k - h) * (-h);
-    idx0 = ((e % NS) + NS) % NS;
-    step = ((k - h) % NS + NS) % NS;
-}
-
-struct ItemSetup {
-    idg_metadata md;
-    int nc;                 // channels in the item
-    int st1, st2;           // stations of the baseline (A_p, A_q)
-    double u0, v0, w0;      // uv(w) of the subgrid centre cell, wavelengths
-    double f_ref;           // reference nu / c of the channel block, 1/m
-};
-
-__device__ __forceinline__ ItemSetup item_setup(const KernelArgs &a, int item, int NS) {
-    ItemSetup s;
-    s.md = a.items[item];
-    s.nc = s.md.channel_end - s.md.channel_begin;
-    s.st1 = a.baselines[2 * s.md.baseline];
-    s.st2 = a.baselines[2 * s.md.baseline + 1];
-    s.u0 = double(s.md.x + NS / 2 - a.grid_size / 2) * a.inv_image_size;
-    s.v0 = double(s.md.y + NS / 2 - a.grid_size / 2) * a.inv_image_size;
-    s.w0 = a.w_offset;
-    s.f_ref = a.frequencies[s.md.channel_begin + s.nc / 2] / kSpeedOfLight;
-    return s;
-}
-
-// B_t and Q_t coefficients (2 pi x wavelengths) of one timestep, formed in fp64.
-__device__ __forceinline__ void timestep_coefficients(const KernelArgs &a, const ItemSetup &s,
-                                                      int t, float4 &cB, float4 &cQ) {
-    const float *p = a.uvw + (int64_t(s.md.baseline) * a.nr_timesteps + t) * 3;
-    const float u = p[0], v = p[1], w = p[2];
-    cB = make_float4(float(kTwoPi * (double(u) * s.f_ref - s.u0)),
-                     float(kTwoPi * (double(v) * s.f_ref - s.v0)),
-                     float(kTwoPi * (double(w) * s.f_ref - s.w0)), 0.0f);
-    cQ = make_float4(float(kTwoPi * double(u)), float(kTwoPi * double(v)),
-                     float(kTwoPi * double(w)), 0.0f);
-}
+constexpr double kTwoPi = dev::kTwoPi;
 
 // ------------------------------------------------------------------------------------------------
 // Gridder: thread -> P pixels (strided by the CTA size so every pixel row is written coalesced);
@@ -144,7 +62,7 @@ __global__ void __launch_bounds__(NS *NS / P, MINB) gridder_kernel(const KernelA
     float *df_s = reinterpret_cast<float *>(coef_s + 2 * (VB + 1));  // [nc]
 
     const int item = a.order[blockIdx.x];
-    const ItemSetup s = item_setup(a, item, NS);
+    const dev::ItemSetup s = dev::item_setup(a, item, NS);
     const idg_metadata &md = s.md;
     const int nc = s.nc;
     const int nvis = md.nr_timesteps * nc;
@@ -160,7 +78,7 @@ __global__ void __launch_bounds__(NS *NS / P, MINB) gridder_kernel(const KernelA
         const int x = pix % NS, y = pix / NS;
         l[k] = float(x - h) * a.cell_l;
         m[k] = float(y - h) * a.cell_l;
-        n[k] = w_term_n(l[k], m[k]);
+        n[k] = dev::w_term_n(l[k], m[k]);
 #pragma unroll
         for (int j = 0; j < 8; ++j) acc[k][j] = 0.0f;
     }
@@ -175,19 +93,19 @@ __global__ void __launch_bounds__(NS *NS / P, MINB) gridder_kernel(const KernelA
         __syncthreads();
         if (contiguous) {
             const float4 *src = reinterpret_cast<const float4 *>(vis0) + 2 * int64_t(e0);
-            for (int i = threadIdx.x; i < 2 * (e1 - e0); i += NT) vis_s[i] = ld_stream(src + i);
+            for (int i = threadIdx.x; i < 2 * (e1 - e0); i += NT) vis_s[i] = dev::ld_stream(src + i);
         } else {
             for (int i = threadIdx.x; i < 2 * (e1 - e0); i += NT) {
                 const int e = e0 + (i >> 1);
                 const int t = e / nc, c = e - t * nc;
                 const float4 *src = reinterpret_cast<const float4 *>(
                     vis0 + int64_t(t) * row + int64_t(md.channel_begin + c) * 4);
-                vis_s[i] = ld_stream(src + (i & 1));
+                vis_s[i] = dev::ld_stream(src + (i & 1));
             }
         }
         for (int t = t_first + int(threadIdx.x); t <= t_last; t += NT) {
             float4 cB, cQ;
-            timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
+            dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
             coef_s[2 * (t - t_first)] = cB;
             coef_s[2 * (t - t_first) + 1] = cQ;
         }
@@ -245,72 +163,14 @@ __global__ void __launch_bounds__(NS *NS / P, MINB) gridder_kernel(const KernelA
     float2 *sub_s = reinterpret_cast<float2 *>(smem);  // [4][NS][NS]
     float2 *tmp_s = sub_s + 4 * NPIX;                  // [4][NS][NS]
     __shared__ float2 tw[NS];
-    init_twiddles<NS>(tw, -1.0f);
-    const float2 *Ap_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st1) * NPIX) * 4;
-    const float2 *Aq_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st2) * NPIX) * 4;
 #pragma unroll
     for (int k = 0; k < P; ++k) {
         const int pix = threadIdx.x + k * NT;
-        const float4 *ap4 = reinterpret_cast<const float4 *>(Ap_base + int64_t(pix) * 4);
-        const float4 *aq4 = reinterpret_cast<const float4 *>(Aq_base + int64_t(pix) * 4);
-        const float4 ap01 = ap4[0], ap23 = ap4[1], aq01 = aq4[0], aq23 = aq4[1];
-        const float2 p0 = make_float2(ap01.x, ap01.y), p1 = make_float2(ap01.z, ap01.w);
-        const float2 p2 = make_float2(ap23.x, ap23.y), p3 = make_float2(ap23.z, ap23.w);
-        const float2 q0 = make_float2(aq01.x, aq01.y), q1 = make_float2(aq01.z, aq01.w);
-        const float2 q2 = make_float2(aq23.x, aq23.y), q3 = make_float2(aq23.z, aq23.w);
-        const float2 s0 = make_float2(acc[k][0], acc[k][1]), s1 = make_float2(acc[k][2], acc[k][3]);
-        const float2 s2 = make_float2(acc[k][4], acc[k][5]), s3 = make_float2(acc[k][6], acc[k][7]);
-        // M = A_p^H S
-        const float2 m0 = cadd(cmulc(p0, s0), cmulc(p2, s2));
-        const float2 m1 = cadd(cmulc(p0, s1), cmulc(p2, s3));
-        const float2 m2 = cadd(cmulc(p1, s0), cmulc(p3, s2));
-        const float2 m3 = cadd(cmulc(p1, s1), cmulc(p3, s3));
-        // R = sph * M A_q   (R-6: adjoint A-term in gridding)
-        const float sph = a.taper[pix];
-        sub_s[0 * NPIX + pix] = cscale(cadd(cmul(m0, q0), cmul(m1, q2)), sph);
-        sub_s[1 * NPIX + pix] = cscale(cadd(cmul(m0, q1), cmul(m1, q3)), sph);
-        sub_s[2 * NPIX + pix] = cscale(cadd(cmul(m2, q0), cmul(m3, q2)), sph);
-        sub_s[3 * NPIX + pix] = cscale(cadd(cmul(m2, q1), cmul(m3, q3)), sph);
+#pragma unroll
+        for (int pol = 0; pol < 4; ++pol) sub_s[pol * NPIX + pix] = make_float2(acc[k][2 * pol], acc[k][2 * pol + 1]);
     }
     __syncthreads();
-    // rows: tmp[pol][y][kx] = sum_x sub[pol][y][x] exp(-2 pi i (kx-h)(x-h)/N~)
-    for (int o = threadIdx.x; o < 4 * NPIX; o += NT) {
-        const int pol = o / NPIX, rem = o - pol * NPIX, y = rem / NS, kx = rem - y * NS;
-        int idx, step;
-        dft_index<NS>(kx, idx, step);
-        const float2 *src = sub_s + pol * NPIX + y * NS;
-        float2 sum = make_float2(0.0f, 0.0f);
-#pragma unroll
-        for (int x = 0; x < NS; ++x) {
-            const float2 w = tw[idx];
-            const float2 v = src[x];
-            sum.x = fmaf(v.x, w.x, fmaf(-v.y, w.y, sum.x));
-            sum.y = fmaf(v.x, w.y, fmaf(v.y, w.x, sum.y));
-            idx += step;
-            idx -= (idx >= NS) ? NS : 0;
-        }
-        tmp_s[o] = sum;
-    }
-    __syncthreads();
-    // columns + adder: G[pol][y_j+ky][x_j+kx] += sum_y tmp[pol][y][kx] exp(-2 pi i (ky-h)(y-h)/N~)
-    for (int o = threadIdx.x; o < 4 * NPIX; o += NT) {
-        const int pol = o / NPIX, rem = o - pol * NPIX, ky = rem / NS, kx = rem - ky * NS;
-        int idx, step;
-        dft_index<NS>(ky, idx, step);
-        const float2 *src = tmp_s + pol * NPIX + kx;
-        float2 sum = make_float2(0.0f, 0.0f);
-#pragma unroll
-        for (int y = 0; y < NS; ++y) {
-            const float2 w = tw[idx];
-            const float2 v = src[y * NS];
-            sum.x = fmaf(v.x, w.x, fmaf(-v.y, w.y, sum.x));
-            sum.y = fmaf(v.x, w.y, fmaf(v.y, w.x, sum.y));
-            idx += step;
-            idx -= (idx >= NS) ? NS : 0;
-        }
-        float2 *dst = a.grid + (int64_t(pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx;
-        red_add(dst, sum);
-    }
+    dev::gridder_epilogue<NS>(a, s, sub_s, tmp_s, tw);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -338,84 +198,22 @@ __global__ void __launch_bounds__(NT, MINB) degridder_kernel(const KernelArgs a)
     __shared__ float2 tw[NS];
 
     const int item = a.order[blockIdx.x];
-    const ItemSetup s = item_setup(a, item, NS);
+    const dev::ItemSetup s = dev::item_setup(a, item, NS);
     const idg_metadata &md = s.md;
     const int nc = s.nc;
 
-    // a6 splitter: sub[pol][ky][kx] = G[pol][y_j+ky][x_j+kx]
-    for (int o = threadIdx.x; o < 4 * NPIX; o += NT) {
-        const int pol = o / NPIX, rem = o - pol * NPIX, ky = rem / NS, kx = rem - ky * NS;
-        sub_s[o] = a.grid[(int64_t(pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx];
-    }
     for (int c = threadIdx.x; c < nc; c += NT)
         df_s[c] = float((a.frequencies[md.channel_begin + c] / kSpeedOfLight) - s.f_ref);
-    init_twiddles<NS>(tw, +1.0f);
-    __syncthreads();
-    // a7 columns: tmp[pol][y][kx] = sum_ky sub[pol][ky][kx] exp(+2 pi i (ky-h)(y-h)/N~)
-    for (int o = threadIdx.x; o < 4 * NPIX; o += NT) {
-        const int pol = o / NPIX, rem = o - pol * NPIX, y = rem / NS, kx = rem - y * NS;
-        int idx, step;
-        dft_index<NS>(y, idx, step);
-        const float2 *src = sub_s + pol * NPIX + kx;
-        float2 sum = make_float2(0.0f, 0.0f);
-#pragma unroll
-        for (int ky = 0; ky < NS; ++ky) {
-            const float2 w = tw[idx];
-            const float2 v = src[ky * NS];
-            sum.x = fmaf(v.x, w.x, fmaf(-v.y, w.y, sum.x));
-            sum.y = fmaf(v.x, w.y, fmaf(v.y, w.x, sum.y));
-            idx += step;
-            idx -= (idx >= NS) ? NS : 0;
-        }
-        tmp_s[o] = sum;
-    }
-    __syncthreads();
-    // a7 rows + Alg. 2 lines 2-3 (taper, A_p S A_q^H) -> pixel records {l, m, n, -}, S
-    const float2 *Ap_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st1) * NPIX) * 4;
-    const float2 *Aq_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st2) * NPIX) * 4;
+    dev::degridder_split_columns<NS>(a, s, sub_s, tmp_s, tw);
+    // a7 rows + Alg. 2 lines 2-3 -> pixel records {l, m, n, -}, S (region A: sub_s is dead now)
     for (int pix = threadIdx.x; pix < NPIX; pix += NT) {
+        float2 r[4];
+        dev::degridder_pixel<NS>(a, s, tmp_s, tw, pix, r);
         const int y = pix / NS, x = pix - y * NS;
-        int idx0, step;
-        dft_index<NS>(x, idx0, step);
-        float2 sv[4];
-#pragma unroll
-        for (int pol = 0; pol < 4; ++pol) {
-            const float2 *src = tmp_s + pol * NPIX + y * NS;
-            float2 sum = make_float2(0.0f, 0.0f);
-            int idx = idx0;
-#pragma unroll
-            for (int kx = 0; kx < NS; ++kx) {
-                const float2 w = tw[idx];
-                const float2 v = src[kx];
-                sum.x = fmaf(v.x, w.x, fmaf(-v.y, w.y, sum.x));
-                sum.y = fmaf(v.x, w.y, fmaf(v.y, w.x, sum.y));
-                idx += step;
-                idx -= (idx >= NS) ? NS : 0;
-            }
-            sv[pol] = sum;
-        }
-        const float4 *ap4 = reinterpret_cast<const float4 *>(Ap_base + int64_t(pix) * 4);
-        const float4 *aq4 = reinterpret_cast<const float4 *>(Aq_base + int64_t(pix) * 4);
-        const float4 ap01 = ap4[0], ap23 = ap4[1], aq01 = aq4[0], aq23 = aq4[1];
-        const float2 p0 = make_float2(ap01.x, ap01.y), p1 = make_float2(ap01.z, ap01.w);
-        const float2 p2 = make_float2(ap23.x, ap23.y), p3 = make_float2(ap23.z, ap23.w);
-        const float2 q0 = make_float2(aq01.x, aq01.y), q1 = make_float2(aq01.z, aq01.w);
-        const float2 q2 = make_float2(aq23.x, aq23.y), q3 = make_float2(aq23.z, aq23.w);
-        // M = A_p S ; R = sph * M A_q^H   (Eq. 1: A_p B A_q^H)
-        const float2 m0 = cadd(cmul(p0, sv[0]), cmul(p1, sv[2]));
-        const float2 m1 = cadd(cmul(p0, sv[1]), cmul(p1, sv[3]));
-        const float2 m2 = cadd(cmul(p2, sv[0]), cmul(p3, sv[2]));
-        const float2 m3 = cadd(cmul(p2, sv[1]), cmul(p3, sv[3]));
-        const float sph = a.taper[pix];
-        const float2 r0 = cscale(cadd(cmul_conj_b(m0, q0), cmul_conj_b(m1, q1)), sph);
-        const float2 r1 = cscale(cadd(cmul_conj_b(m0, q2), cmul_conj_b(m1, q3)), sph);
-        const float2 r2 = cscale(cadd(cmul_conj_b(m2, q0), cmul_conj_b(m3, q1)), sph);
-        const float2 r3 = cscale(cadd(cmul_conj_b(m2, q2), cmul_conj_b(m3, q3)), sph);
         const float l = float(x - h) * a.cell_l, m = float(y - h) * a.cell_l;
-        // region A is rewritten: sub_s is dead after the column pass (barrier above)
-        pix_s[3 * pix + 0] = make_float4(l, m, w_term_n(l, m), 0.0f);
-        pix_s[3 * pix + 1] = make_float4(r0.x, r0.y, r1.x, r1.y);
-        pix_s[3 * pix + 2] = make_float4(r2.x, r2.y, r3.x, r3.y);
+        pix_s[3 * pix + 0] = make_float4(l, m, dev::w_term_n(l, m), 0.0f);
+        pix_s[3 * pix + 1] = make_float4(r[0].x, r[0].y, r[1].x, r[1].y);
+        pix_s[3 * pix + 2] = make_float4(r[2].x, r[2].y, r[3].x, r[3].y);
     }
     __syncthreads();
 
@@ -428,7 +226,7 @@ __global__ void __launch_bounds__(NT, MINB) degridder_kernel(const KernelArgs a)
         const int t = slot / groups;
         const int c0 = (slot - t * groups) * V;
         float4 cB, cQ;
-        timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
+        dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
         float df[V];
         float acc[V][8];
 #pragma unroll
@@ -478,20 +276,12 @@ __global__ void __launch_bounds__(NT, MINB) degridder_kernel(const KernelArgs a)
     }
 }
 
-template <typename K>
-cudaError_t prepare(K kernel, size_t smem) {
-    cudaError_t err = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-    if (err != cudaSuccess) return err;
-    return cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                int(cudaSharedmemCarveoutMaxShared));
-}
-
 template <int NS, int P, int MINB>
 cudaError_t launch_gridder_t(const KernelArgs &a, cudaStream_t st) {
     constexpr int NT = NS * NS / P;
     static_assert(NS * NS % (P * 32) == 0, "pixels per thread must give whole warps");
     const size_t smem = gridder_smem_bytes(NS, a.max_channels_in_item);
-    cudaError_t err = prepare(gridder_kernel<NS, P, MINB>, smem);
+    cudaError_t err = dev::prepare(gridder_kernel<NS, P, MINB>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("gridder", st);
     gridder_kernel<NS, P, MINB><<<unsigned(a.nr_items), NT, smem, st>>>(a);
@@ -501,29 +291,23 @@ cudaError_t launch_gridder_t(const KernelArgs &a, cudaStream_t st) {
 template <int NS, int V, int NT, int MINB>
 cudaError_t launch_degridder_t(const KernelArgs &a, cudaStream_t st) {
     const size_t smem = degridder_smem_bytes(NS, a.max_channels_in_item);
-    cudaError_t err = prepare(degridder_kernel<NS, V, NT, MINB>, smem);
+    cudaError_t err = dev::prepare(degridder_kernel<NS, V, NT, MINB>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("degridder", st);
     degridder_kernel<NS, V, NT, MINB><<<unsigned(a.nr_items), NT, smem, st>>>(a);
     return cudaGetLastError();
 }
 
-using Launcher = cudaError_t (*)(const KernelArgs &, cudaStream_t);
-struct Variant {
-    int ns, v;            // subgrid size; pixels (gridder) or channels (degridder) per thread
-    const char *name;
-    Launcher fn;
-};
-
-// Launch-shape variants (tuned on B200 with scripts/tune.py; the first entry per (NS, V) is the default).
-#define GV(NS, P, MB) {NS, 0, "gridder<" #NS ",P" #P ",minB" #MB ">", launch_gridder_t<NS, P, MB>}
+// SIMT launch-shape variants (first entry per (NS, V) is the SIMT default; tuned with scripts/tune.py).
+// v = channels per thread for the degridder (every item's channel count must be a multiple of v).
+#define GV(NS, P, MB) {NS, 0, kSimt, "gridder<" #NS ",P" #P ",minB" #MB ">", launch_gridder_t<NS, P, MB>}
 const Variant kGridderVariants[] = {
     GV(24, 6, 4), GV(24, 6, 5), GV(24, 6, 6), GV(24, 3, 3), GV(24, 3, 4), GV(24, 2, 4), GV(24, 9, 3),
     GV(32, 4, 2), GV(32, 8, 3), GV(32, 8, 4), GV(32, 4, 3), GV(32, 16, 4),
     GV(16, 4, 4), GV(16, 4, 6), GV(16, 2, 4), GV(16, 8, 6),
 };
 #undef GV
-#define DV(NS, V, NT, MB) {NS, V, "degridder<" #NS ",V" #V ",T" #NT ",minB" #MB ">", launch_degridder_t<NS, V, NT, MB>}
+#define DV(NS, V, NT, MB) {NS, V, kSimt, "degridder<" #NS ",V" #V ",T" #NT ",minB" #MB ">", launch_degridder_t<NS, V, NT, MB>}
 #define DV_ALL(NS) DV(NS, 8, 128, 4), DV(NS, 8, 128, 3), DV(NS, 8, 256, 1), DV(NS, 8, 256, 2), \
     DV(NS, 8, 64, 6), DV(NS, 8, 64, 8), DV(NS, 4, 128, 4), DV(NS, 4, 256, 3), DV(NS, 4, 128, 6), \
     DV(NS, 2, 128, 6), DV(NS, 1, 128, 6)
@@ -531,48 +315,62 @@ const Variant kDegridderVariants[] = {DV_ALL(24), DV_ALL(32), DV_ALL(16)};
 #undef DV_ALL
 #undef DV
 
-// Variant choice: default = first match; env IDG_GRIDDER_VARIANT / IDG_DEGRIDDER_VARIANT = name
-// overrides (tuning only).
-template <size_t K>
-const Variant *pick(const Variant (&table)[K], int ns, int v, const char *env) {
+bool eligible(const Variant &var, int ns, int channel_gcd) {
+    if (var.ns != ns) return false;
+    if (var.kind == kTensor) return var.v == 0 || channel_gcd % var.v == 0;
+    return var.v == 0 || channel_gcd % var.v == 0;
+}
+
+// Variant choice.  Default: the first eligible tensor-core variant, else the first eligible SIMT
+// variant (for the SIMT degridder: the one with the largest channels-per-thread).  The environment
+// variable `env` (IDG_GRIDDER_VARIANT / IDG_DEGRIDDER_VARIANT) may name any eligible variant (tuning).
+const Variant *pick(const Variant *simt, int nsimt, const Variant *tc, int ntc, int ns, int channel_gcd,
+                    const char *env) {
     const char *want = std::getenv(env);
-    const Variant *first = nullptr;
-    for (const Variant &var : table) {
-        if (var.ns != ns) continue;
-        // an override may use fewer channels per thread than the default, as long as it divides it
-        const bool valid = (v == 0) ? var.v == 0 : (var.v > 0 && v % var.v == 0);
-        if (valid && want && std::strcmp(want, var.name) == 0) return &var;
-        if (!first && var.v == v) first = &var;
+    if (want && *want) {
+        for (int i = 0; i < ntc; ++i)
+            if (eligible(tc[i], ns, channel_gcd) && std::strcmp(want, tc[i].name) == 0) return &tc[i];
+        for (int i = 0; i < nsimt; ++i)
+            if (eligible(simt[i], ns, channel_gcd) && std::strcmp(want, simt[i].name) == 0) return &simt[i];
     }
-    return first;
+    if (!(want && std::strcmp(want, "simt") == 0))
+        for (int i = 0; i < ntc; ++i)
+            if (eligible(tc[i], ns, channel_gcd)) return &tc[i];
+    const Variant *best = nullptr;
+    for (int i = 0; i < nsimt; ++i)
+        if (eligible(simt[i], ns, channel_gcd) && (!best || simt[i].v > best->v)) best = &simt[i];
+    return best;
 }
 
 }  // namespace
 
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
-    const Variant *var = pick(kGridderVariants, a.subgrid_size, 0, "IDG_GRIDDER_VARIANT");
+    int ntc = 0;
+    const Variant *tc = tc_gridder_variants(&ntc);
+    const Variant *var = pick(kGridderVariants, int(std::size(kGridderVariants)), tc, ntc, a.subgrid_size,
+                              a.channel_gcd, "IDG_GRIDDER_VARIANT");
     return var ? var->fn(a, s) : cudaErrorInvalidValue;
 }
 
-// The channel count of every item must be a multiple of V (the host picks V from the plan).
-int degridder_channels_per_thread(int channel_gcd) {
-    if (channel_gcd % 8 == 0) return 8;
-    if (channel_gcd % 4 == 0) return 4;
-    if (channel_gcd % 2 == 0) return 2;
-    return 1;
-}
-
-cudaError_t launch_degridder_v(const KernelArgs &a, int V, cudaStream_t s) {
+cudaError_t launch_degridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
-    const Variant *var = pick(kDegridderVariants, a.subgrid_size, V, "IDG_DEGRIDDER_VARIANT");
+    int ntc = 0;
+    const Variant *tc = tc_degridder_variants(&ntc);
+    const Variant *var = pick(kDegridderVariants, int(std::size(kDegridderVariants)), tc, ntc, a.subgrid_size,
+                              a.channel_gcd, "IDG_DEGRIDDER_VARIANT");
     return var ? var->fn(a, s) : cudaErrorInvalidValue;
 }
 
 const char *variant_names(int which) {
     static std::string g, d;
     if (g.empty()) {
+        int n = 0;
+        const Variant *tc = tc_gridder_variants(&n);
+        for (int i = 0; i < n; ++i) g += std::string(tc[i].name) + "\n";
         for (const Variant &v : kGridderVariants) g += std::string(v.name) + "\n";
+        tc = tc_degridder_variants(&n);
+        for (int i = 0; i < n; ++i) d += std::string(tc[i].name) + "\n";
         for (const Variant &v : kDegridderVariants) d += std::string(v.name) + "\n";
     }
     return which == 0 ? g.c_str() : d.c_str();

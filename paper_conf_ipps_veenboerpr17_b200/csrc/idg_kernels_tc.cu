@@ -1,0 +1,428 @@
+// idg_kernels_tc.cu -- tensor-core sm_100a gridder and degridder (Veenboer et al., IPDPS 2017).
+//
+// The pixel x visibility phasor contraction of Alg. 1 / Alg. 2 is a dense complex matrix product:
+//     gridder    S[pixel][pol]  = sum_v  Phi[pixel][v]     V[v][pol]      (Phi = exp(+i phi))
+//     degridder  V[v][pol]      = sum_p  Phi*[v][p]        S[p][pol]
+// written as a real product with K = 2 x (visibilities or pixels) and N = 8 = 4 pols x (re, im):
+//     A[m][2k] = cos phi, A[m][2k+1] = sin phi;  B[2k][2pol], B[2k+1][2pol], ... encode the complex MAC
+// so one warp-level mma.m16n8k16 covers 16 pixels (or visibilities) x 8 visibilities (or pixels) =
+// 128 (pixel, visibility) pairs.  The 16 multiply-adds per pair of the paper move to the tensor
+// cores; the ALUs keep the phase (1 FMA), the sincos (FMUL + MUFU.SIN + MUFU.COS) and the
+// operand split.  Precision: every operand is split into f16 hi + lo (x = hi + lo to ~22 bits) and the
+// product is formed as hi*hi + hi*lo + lo*hi with fp32 accumulation (three mma per tile).  f16 range:
+// visibilities / subgrid pixels are scaled by a power of two per batch / per item (exact).
+//
+// Operand layouts (PTX mma.m16n8k16, g = lane/4, q = lane%4):
+//   A regs: {A[g][2q..2q+1]}, {A[g+8][2q..]}, {A[g][2q+8..]}, {A[g+8][2q+8..]}  -> thread computes the
+//           phasors of (row g, k-slot q), (row g+8, q), (row g, q+4), (row g+8, q+4)
+//   B regs: {B[2q..2q+1][g]}, {B[2q+8..2q+9][g]}  -> prepared once per k-block in shared memory
+//   D regs: D[g][2q..2q+1], D[g+8][2q..2q+1]      -> (row g, pol q, re/im), (row g+8, pol q, re/im)
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+
+#include "idg_device.cuh"
+#include "idg_internal.h"
+
+namespace idg {
+namespace {
+
+using dev::ItemSetup;
+
+__device__ __forceinline__ uint32_t h2_bits(__half2 h) { return *reinterpret_cast<uint32_t *>(&h); }
+
+// (x, y) -> f16x2 hi = rn(x, y) and lo = rn(x - hi, y - hi): x = hi + lo to ~22 significant bits.
+__device__ __forceinline__ void split2(float x, float y, uint32_t &hi, uint32_t &lo) {
+    const __half2 h = __floats2half2_rn(x, y);
+    const float2 hf = __half22float2(h);
+    const __half2 l = __floats2half2_rn(x - hf.x, y - hf.y);
+    hi = h2_bits(h);
+    lo = h2_bits(l);
+}
+
+__device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
+                                         uint32_t b0, uint32_t b1) {
+    asm("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+}
+
+// The three split products of one tile: D += Ahi Bhi + Ahi Blo + Alo Bhi.
+__device__ __forceinline__ void mma3(float (&d)[4], const uint32_t (&ah)[4], const uint32_t (&al)[4],
+                                     const uint4 &b) {
+    mma16816(d, ah[0], ah[1], ah[2], ah[3], b.x, b.y);
+    mma16816(d, ah[0], ah[1], ah[2], ah[3], b.z, b.w);
+    mma16816(d, al[0], al[1], al[2], al[3], b.x, b.y);
+}
+
+// Power-of-two scale s with max * s in [2^13, 2^14) (f16 max is 65504); 1 for max == 0.
+__device__ __forceinline__ float pow2_scale(float mx) {
+    if (!(mx > 0.0f)) return 1.0f;
+    int e = int((__float_as_uint(mx) >> 23) & 0xff) - 127;
+    int sexp = min(max(13 - e, -120), 120);
+    return __uint_as_float(uint32_t(127 + sexp) << 23);
+}
+
+template <int WARPS>
+__device__ __forceinline__ float block_max(float v, float *red_s) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0) red_s[threadIdx.x >> 5] = v;
+    __syncthreads();
+    float m = red_s[0];
+#pragma unroll
+    for (int w = 1; w < WARPS; ++w) m = fmaxf(m, red_s[w]);
+    return m;
+}
+
+__device__ __forceinline__ float4 abs_max4(float4 v, float m) {
+    return make_float4(fmaxf(m, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w)))), 0, 0, 0);
+}
+
+// ------------------------------------------------------------------------------------------------
+// Tensor-core gridder.  One CTA per work item; WARPS warps x MT m-tiles x 16 pixels = N~^2.
+// k-block = 8 visibilities = 8 consecutive channels of one timestep (requires C~ % 8 == 0).
+// ------------------------------------------------------------------------------------------------
+constexpr int kTcBatchKB = 64;  // k-blocks per shared-memory batch (512 visibilities)
+
+inline size_t gridder_tc_smem_bytes(int NS, int max_channels) {
+    const size_t kbb = kTcBatchKB;
+    const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + kbb * 4 * 8 /*df*/ +
+                        (kbb + 1) * 32 /*coef*/ + size_t(max_channels) * 4;
+    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2);
+    return std::max(main, epi) + 16;
+}
+
+template <int NS, int WARPS, int MT, int MINB>
+__global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const KernelArgs a) {
+    constexpr int NT = WARPS * 32;
+    constexpr int NPIX = NS * NS;
+    static_assert(WARPS * MT * 16 == NPIX, "warps x m-tiles x 16 must cover the subgrid");
+    constexpr int h = NS / 2;
+    constexpr int KBB = kTcBatchKB;
+    constexpr int VB = KBB * 8;
+    extern __shared__ __align__(16) unsigned char smem[];
+    float4 *raw_s = reinterpret_cast<float4 *>(smem);                // [VB][2]
+    uint4 *frag_s = reinterpret_cast<uint4 *>(raw_s + 2 * VB);       // [KBB][32]
+    float2 *dfk_s = reinterpret_cast<float2 *>(frag_s + KBB * 32);   // [KBB][4]
+    float4 *coef_s = reinterpret_cast<float4 *>(dfk_s + KBB * 4);    // [KBB+1][2]
+    float *df_s = reinterpret_cast<float *>(coef_s + 2 * (KBB + 1)); // [nc]
+    __shared__ float red_s[WARPS];
+    __shared__ float2 tw[NS];
+
+    const int item = a.order[blockIdx.x];
+    const ItemSetup s = dev::item_setup(a, item, NS);
+    const idg_metadata &md = s.md;
+    const int nc = s.nc;
+    const int kpt = nc >> 3;                     // k-blocks per timestep
+    const int nkb = md.nr_timesteps * kpt;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
+
+    for (int c = threadIdx.x; c < nc; c += NT)
+        df_s[c] = float((a.frequencies[md.channel_begin + c] / kSpeedOfLight) - s.f_ref);
+
+    float pl[MT][2], pm[MT][2], pn[MT][2], acc[MT][4];
+#pragma unroll
+    for (int i = 0; i < MT; ++i) {
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            const int pix = (warp * MT + i) * 16 + g + 8 * r;
+            const int x = pix % NS, y = pix / NS;
+            pl[i][r] = float(x - h) * a.cell_l;
+            pm[i][r] = float(y - h) * a.cell_l;
+            pn[i][r] = dev::w_term_n(pl[i][r], pm[i][r]);
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
+    }
+    float cur_scale = 0.0f;
+
+    const int64_t row = int64_t(a.nr_channels) * 4;  // float2 per timestep
+    const float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
+                         int64_t(md.channel_begin) * 4;
+
+    for (int kb0 = 0; kb0 < nkb; kb0 += KBB) {
+        const int kb1 = min(kb0 + KBB, nkb);
+        const int nvb = (kb1 - kb0) * 8;
+        const int t_first = kb0 / kpt, t_last = (kb1 - 1) / kpt;
+        __syncthreads();  // previous batch fully consumed
+        // (1) raw visibilities of k-blocks [kb0, kb1)
+        for (int i = threadIdx.x; i < 2 * nvb; i += NT) {
+            const int j = i >> 1;
+            const int kb = kb0 + (j >> 3);
+            const int t = kb / kpt;
+            const int c = (kb - t * kpt) * 8 + (j & 7);
+            raw_s[i] = dev::ld_stream(reinterpret_cast<const float4 *>(vis0 + int64_t(t) * row + c * 4) + (i & 1));
+        }
+        // (2) per-timestep phase coefficients (fp64 -> fp32)
+        for (int t = t_first + int(threadIdx.x); t <= t_last; t += NT) {
+            float4 cB, cQ;
+            dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
+            coef_s[2 * (t - t_first)] = cB;
+            coef_s[2 * (t - t_first) + 1] = cQ;
+        }
+        // (3) channel offsets of the two k-slots q, q+4 of every k-block
+        for (int i = threadIdx.x; i < (kb1 - kb0) * 4; i += NT) {
+            const int kb = kb0 + (i >> 2);
+            const int c = (kb % kpt) * 8 + (i & 3);
+            dfk_s[i] = make_float2(df_s[c], df_s[c + 4]);
+        }
+        __syncthreads();
+        // (4) f16 range: power-of-two scale from the batch maximum; never increase the running scale
+        float mx = 0.0f;
+        for (int i = threadIdx.x; i < 2 * nvb; i += NT) mx = abs_max4(raw_s[i], mx).x;
+        const float bscale = pow2_scale(block_max<WARPS>(mx, red_s));
+        if (cur_scale == 0.0f) {
+            cur_scale = bscale;
+        } else if (bscale < cur_scale) {
+            const float f = bscale / cur_scale;  // exact power of two
+#pragma unroll
+            for (int i = 0; i < MT; ++i)
+#pragma unroll
+                for (int j = 0; j < 4; ++j) acc[i][j] *= f;
+            cur_scale = bscale;
+        }
+        // (5) B fragments: entry (k-block, lane): column g = 2 pol + im, k-slots q and q+4
+        for (int i = threadIdx.x; i < (kb1 - kb0) * 32; i += NT) {
+            const int kbl = i >> 5, ln = i & 31, gg = ln >> 2, qq = ln & 3;
+            const int pol = gg >> 1, im = gg & 1;
+            uint32_t hi[2], lo[2];
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const float4 v4 = raw_s[2 * (kbl * 8 + qq + 4 * r) + (pol >> 1)];
+                const float vr = ((pol & 1) ? v4.z : v4.x) * cur_scale;
+                const float vi = ((pol & 1) ? v4.w : v4.y) * cur_scale;
+                // column 2pol:   rows (cos, sin) -> ( Vre, -Vim );  column 2pol+1: ( Vim, Vre )
+                split2(im ? vi : vr, im ? vr : -vi, hi[r], lo[r]);
+            }
+            frag_s[i] = make_uint4(hi[0], hi[1], lo[0], lo[1]);
+        }
+        __syncthreads();
+        // (6) the contraction: per k-block, MT tiles x (4 phasors + 3 mma) per thread
+        int cur_t = -1;
+        float Bv[MT][2], Qv[MT][2];
+        for (int kb = kb0; kb < kb1; ++kb) {
+            const int t = kb / kpt;
+            if (t != cur_t) {
+                cur_t = t;
+                const float4 cB = coef_s[2 * (t - t_first)], cQ = coef_s[2 * (t - t_first) + 1];
+#pragma unroll
+                for (int i = 0; i < MT; ++i)
+#pragma unroll
+                    for (int r = 0; r < 2; ++r) {
+                        Bv[i][r] = fmaf(cB.x, pl[i][r], fmaf(cB.y, pm[i][r], cB.z * pn[i][r]));
+                        Qv[i][r] = fmaf(cQ.x, pl[i][r], fmaf(cQ.y, pm[i][r], cQ.z * pn[i][r]));
+                    }
+            }
+            const uint4 bf = frag_s[(kb - kb0) * 32 + lane];
+            const float2 df = dfk_s[(kb - kb0) * 4 + q];
+#pragma unroll
+            for (int i = 0; i < MT; ++i) {
+                float sn[4], cs[4];
+                __sincosf(fmaf(df.x, Qv[i][0], Bv[i][0]), &sn[0], &cs[0]);  // row g,   slot q
+                __sincosf(fmaf(df.x, Qv[i][1], Bv[i][1]), &sn[1], &cs[1]);  // row g+8, slot q
+                __sincosf(fmaf(df.y, Qv[i][0], Bv[i][0]), &sn[2], &cs[2]);  // row g,   slot q+4
+                __sincosf(fmaf(df.y, Qv[i][1], Bv[i][1]), &sn[3], &cs[3]);  // row g+8, slot q+4
+                uint32_t ah[4], al[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) split2(cs[j], sn[j], ah[j], al[j]);
+                mma3(acc[i], ah, al, bf);
+            }
+        }
+    }
+
+    // ---- epilogue: D fragments -> sub_s[pol][pixel], then a3 + a4 + a5 ---------------------------
+    __syncthreads();
+    float2 *sub_s = reinterpret_cast<float2 *>(smem);
+    float2 *tmp_s = sub_s + 4 * NPIX;
+    const float inv = cur_scale > 0.0f ? 1.0f / cur_scale : 1.0f;
+#pragma unroll
+    for (int i = 0; i < MT; ++i) {
+        const int p0 = (warp * MT + i) * 16 + g;
+        sub_s[q * NPIX + p0] = make_float2(acc[i][0] * inv, acc[i][1] * inv);
+        sub_s[q * NPIX + p0 + 8] = make_float2(acc[i][2] * inv, acc[i][3] * inv);
+    }
+    __syncthreads();
+    dev::gridder_epilogue<NS>(a, s, sub_s, tmp_s, tw);
+}
+
+// ------------------------------------------------------------------------------------------------
+// Tensor-core degridder.  One CTA per work item.  Prologue (a6-a8) leaves the corrected subgrid as
+// B fragments (k-block = 8 pixels) + per-pixel {l, m, n}; m-tile = 16 consecutive visibilities of
+// the item (flattened (t, c) order); each warp takes MT tiles at a time over all k-blocks.
+// ------------------------------------------------------------------------------------------------
+inline size_t degridder_tc_smem_bytes(int NS) {
+    const size_t npix = size_t(NS) * NS;
+    return npix * 64 /*sub+tmp | frag*/ + npix * 16 /*lmn*/ + 16;
+}
+
+template <int NS, int WARPS, int MT, int MINB>
+__global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const KernelArgs a) {
+    constexpr int NT = WARPS * 32;
+    constexpr int NPIX = NS * NS;
+    constexpr int NKB = NPIX / 8;
+    constexpr int PPT = (NPIX + NT - 1) / NT;
+    constexpr int h = NS / 2;
+    static_assert(NPIX % 8 == 0, "pixels per k-block");
+    extern __shared__ __align__(16) unsigned char smem[];
+    float2 *sub_s = reinterpret_cast<float2 *>(smem);                     // [4][NS][NS]
+    float2 *tmp_s = sub_s + 4 * NPIX;                                     // [4][NS][NS]
+    uint4 *frag_s = reinterpret_cast<uint4 *>(smem);                      // [NKB][32] (after prologue)
+    float4 *lmn_s = reinterpret_cast<float4 *>(smem + size_t(NPIX) * 64); // [NPIX]
+    __shared__ float red_s[WARPS];
+    __shared__ float2 tw[NS];
+
+    const int item = a.order[blockIdx.x];
+    const ItemSetup s = dev::item_setup(a, item, NS);
+    const idg_metadata &md = s.md;
+    const int nc = s.nc;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
+
+    dev::degridder_split_columns<NS>(a, s, sub_s, tmp_s, tw);
+    float2 rr[PPT][4];
+    float mx = 0.0f;
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) {
+        const int pix = threadIdx.x + i * NT;
+        if (pix < NPIX) {
+            dev::degridder_pixel<NS>(a, s, tmp_s, tw, pix, rr[i]);
+#pragma unroll
+            for (int p = 0; p < 4; ++p) mx = fmaxf(mx, fmaxf(fabsf(rr[i][p].x), fabsf(rr[i][p].y)));
+            const int y = pix / NS, x = pix - y * NS;
+            const float l = float(x - h) * a.cell_l, m = float(y - h) * a.cell_l;
+            lmn_s[pix] = make_float4(l, m, dev::w_term_n(l, m), 0.0f);
+        }
+    }
+    const float scale = pow2_scale(block_max<WARPS>(mx, red_s));  // barriers: tmp_s reads are done
+    const float inv = 1.0f / scale;
+    uint32_t *frag_w = reinterpret_cast<uint32_t *>(frag_s);
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) {
+        const int pix = threadIdx.x + i * NT;
+        if (pix < NPIX) {
+            const int kb = pix >> 3, slot = pix & 7, qq = slot & 3, half = slot >> 2;
+#pragma unroll
+            for (int gg = 0; gg < 8; ++gg) {
+                const int pol = gg >> 1;
+                const float sr = rr[i][pol].x * scale, si = rr[i][pol].y * scale;
+                uint32_t hi, lo;
+                // V += S exp(-i phi): column 2pol rows (cos, sin) -> (Sre, Sim); column 2pol+1 -> (Sim, -Sre)
+                split2((gg & 1) ? si : sr, (gg & 1) ? -sr : si, hi, lo);
+                const int e = (kb * 32 + gg * 4 + qq) * 4;
+                frag_w[e + half] = hi;
+                frag_w[e + 2 + half] = lo;
+            }
+        }
+    }
+    __syncthreads();
+
+    const int nvis = md.nr_timesteps * nc;
+    const int ntiles = (nvis + 15) >> 4;
+    const int64_t row = int64_t(a.nr_channels) * 4;
+    float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
+                   int64_t(md.channel_begin) * 4;
+    for (int tile0 = warp * MT; tile0 < ntiles; tile0 += WARPS * MT) {
+        float cu[MT][2], cv[MT][2], cw[MT][2], acc[MT][4];
+#pragma unroll
+        for (int i = 0; i < MT; ++i) {
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const int v = (tile0 + i) * 16 + g + 8 * r;
+                cu[i][r] = cv[i][r] = cw[i][r] = 0.0f;
+                if (v < nvis) {
+                    const int t = v / nc, c = v - t * nc;
+                    const float *p = a.uvw + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset + t) * 3;
+                    const double f = a.frequencies[md.channel_begin + c] / kSpeedOfLight;
+                    cu[i][r] = float(dev::kTwoPi * (double(p[0]) * f - s.u0));
+                    cv[i][r] = float(dev::kTwoPi * (double(p[1]) * f - s.v0));
+                    cw[i][r] = float(dev::kTwoPi * (double(p[2]) * f - s.w0));
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
+        }
+#pragma unroll 2
+        for (int kb = 0; kb < NKB; ++kb) {
+            const uint4 bf = frag_s[kb * 32 + lane];
+            const float4 x0 = lmn_s[kb * 8 + q], x1 = lmn_s[kb * 8 + q + 4];
+#pragma unroll
+            for (int i = 0; i < MT; ++i) {
+                float sn[4], cs[4];
+                __sincosf(fmaf(cu[i][0], x0.x, fmaf(cv[i][0], x0.y, cw[i][0] * x0.z)), &sn[0], &cs[0]);
+                __sincosf(fmaf(cu[i][1], x0.x, fmaf(cv[i][1], x0.y, cw[i][1] * x0.z)), &sn[1], &cs[1]);
+                __sincosf(fmaf(cu[i][0], x1.x, fmaf(cv[i][0], x1.y, cw[i][0] * x1.z)), &sn[2], &cs[2]);
+                __sincosf(fmaf(cu[i][1], x1.x, fmaf(cv[i][1], x1.y, cw[i][1] * x1.z)), &sn[3], &cs[3]);
+                uint32_t ah[4], al[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) split2(cs[j], sn[j], ah[j], al[j]);
+                mma3(acc[i], ah, al, bf);
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < MT; ++i) {
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const int v = (tile0 + i) * 16 + g + 8 * r;
+                if (v < nvis) {
+                    const int t = v / nc, c = v - t * nc;
+                    vis0[int64_t(t) * row + c * 4 + q] = make_float2(acc[i][2 * r] * inv, acc[i][2 * r + 1] * inv);
+                }
+            }
+        }
+    }
+}
+
+template <int NS, int WARPS, int MT, int MINB>
+cudaError_t launch_gridder_tc(const KernelArgs &a, cudaStream_t st) {
+    const size_t smem = gridder_tc_smem_bytes(NS, a.max_channels_in_item);
+    cudaError_t err = dev::prepare(gridder_tc_kernel<NS, WARPS, MT, MINB>, smem);
+    if (err != cudaSuccess) return err;
+    LaunchScope scope("gridder", st);
+    gridder_tc_kernel<NS, WARPS, MT, MINB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+template <int NS, int WARPS, int MT, int MINB>
+cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
+    const size_t smem = degridder_tc_smem_bytes(NS);
+    cudaError_t err = dev::prepare(degridder_tc_kernel<NS, WARPS, MT, MINB>, smem);
+    if (err != cudaSuccess) return err;
+    LaunchScope scope("degridder", st);
+    degridder_tc_kernel<NS, WARPS, MT, MINB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+#define TG(NS, W, MT, MB) \
+    {NS, 8, kTensor, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB>}
+const Variant kTcGridder[] = {
+    TG(24, 6, 6, 2), TG(24, 12, 3, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
+    TG(32, 8, 8, 2), TG(32, 16, 4, 1), TG(32, 4, 16, 3), TG(32, 16, 4, 2),
+    TG(16, 4, 4, 4), TG(16, 8, 2, 3), TG(16, 16, 1, 2),
+};
+#undef TG
+#define TD(NS, W, MT, MB) \
+    {NS, 0, kTensor, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>}
+const Variant kTcDegridder[] = {
+    TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 2, 3), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
+    TD(32, 8, 4, 2), TD(32, 4, 4, 3), TD(32, 8, 8, 1), TD(32, 16, 2, 1),
+    TD(16, 8, 4, 2), TD(16, 4, 4, 4), TD(16, 8, 2, 3),
+};
+#undef TD
+
+}  // namespace
+
+const Variant *tc_gridder_variants(int *n) {
+    *n = int(sizeof(kTcGridder) / sizeof(kTcGridder[0]));
+    return kTcGridder;
+}
+
+const Variant *tc_degridder_variants(int *n) {
+    *n = int(sizeof(kTcDegridder) / sizeof(kTcDegridder[0]));
+    return kTcDegridder;
+}
+
+}  // namespace idg

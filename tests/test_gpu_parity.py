@@ -64,23 +64,34 @@ CASES = [
     ("lofar", dict(T=640, nr_stations=5), None, "spheroidal"),       # N~=24, N=2048, 16 ch
     ("lofar_dde", dict(T=512, nr_stations=5), None, "spheroidal"),   # + random A-terms, w0
     ("ska", dict(T=384, nr_stations=4), None, "spheroidal"),         # N~=32, N=8192, 32 ch
+    ("predict", dict(T=256, nr_stations=4, C=8), None, "spheroidal"),  # N~=32, 8 ch: one k-block/timestep
+    ("small_dde", dict(C=24, C_block=8), None, "spheroidal"),       # 3 channel blocks of 8
 ]
 
 
+@pytest.fixture(params=["default", "simt"])
+def kind(request, monkeypatch):
+    """default = tensor-core kernels where eligible; simt = the paper-structured CUDA-core kernels."""
+    if request.param == "simt":
+        monkeypatch.setenv("IDG_GRIDDER_VARIANT", "simt")
+        monkeypatch.setenv("IDG_DEGRIDDER_VARIANT", "simt")
+    return request.param
+
+
 @pytest.mark.parametrize("name,kw,aterm,taper", CASES)
-def test_grid_matches_oracle(name, kw, aterm, taper):
+def test_grid_matches_oracle(name, kw, aterm, taper, kind):
     obs = idgsynth.make_observation(name, **kw)
     vis, aterms, tap = _inputs(obs, aterm, taper)
     items, _ = oracle.plan(obs)
     ref = oracle.grid(obs, items, vis, aterms, tap)
     got = gpu_grid(obs, vis, aterms, tap).cpu().numpy()
     err = rel_rms(got, ref)
-    print(f"grid {name} {kw}: rel rms {err:.3e}")
+    print(f"grid[{kind}] {name} {kw}: rel rms {err:.3e}")
     assert err <= TOL, err
 
 
 @pytest.mark.parametrize("name,kw,aterm,taper", CASES)
-def test_degrid_matches_oracle(name, kw, aterm, taper):
+def test_degrid_matches_oracle(name, kw, aterm, taper, kind):
     obs = idgsynth.make_observation(name, **kw)
     _, aterms, tap = _inputs(obs, aterm, taper)
     G = idgsynth.make_grid(obs)
@@ -88,11 +99,11 @@ def test_degrid_matches_oracle(name, kw, aterm, taper):
     ref = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, G, aterms, tap))
     got = gpu_degrid(obs, G, aterms, tap).cpu().numpy()
     err = rel_rms(got, ref)
-    print(f"degrid {name} {kw}: rel rms {err:.3e}")
+    print(f"degrid[{kind}] {name} {kw}: rel rms {err:.3e}")
     assert err <= TOL, err
 
 
-def test_grid_accumulates_and_degrid_zeroes_dropped():
+def test_grid_accumulates_and_degrid_zeroes_dropped(kind):
     import dataclasses
     obs = idgsynth.make_observation("small_dde")
     obs = dataclasses.replace(obs, image_size=obs.image_size * 6)     # long baselines fall off the grid
@@ -118,7 +129,7 @@ def _inner_t(a, b):
 
 
 @pytest.mark.parametrize("name", ["lofar_dde", "lofar"])
-def test_full_size_adjoint_and_sampled_items(name):
+def test_full_size_adjoint_and_sampled_items(name, kind):
     """Full LOFAR-shaped set in the bench launch configuration: <degrid(G),V> = <G,grid(V)> on the GPU,
     and degridded visibilities of sampled work items against the oracle computing just those items."""
     obs = idgsynth.make_observation(name)
