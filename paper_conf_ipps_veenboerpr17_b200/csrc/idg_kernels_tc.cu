@@ -202,7 +202,14 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
             frag_s[i] = make_uint4(hi[0], hi[1], lo[0], lo[1]);
         }
         __syncthreads();
-        // (6) the contraction: per k-block, MT tiles x (4 phasors + 3 mma) per thread
+        // (6) the contraction: per k-block, MT tiles x (4 phasors + 3 mma) per thread.  Each batch
+        //     accumulates into a fresh fragment that is then added in fp32: the tensor-core
+        //     accumulation error grows with the batch (512 visibilities), not with the whole item.
+        float part[MT][4];
+#pragma unroll
+        for (int i = 0; i < MT; ++i)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) part[i][j] = 0.0f;
         int cur_t = -1;
         float Bv[MT][2], Qv[MT][2];
         for (int kb = kb0; kb < kb1; ++kb) {
@@ -230,9 +237,13 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
                 uint32_t ah[4], al[4];
 #pragma unroll
                 for (int j = 0; j < 4; ++j) split2(cs[j], sn[j], ah[j], al[j]);
-                mma3(acc[i], ah, al, bf);
+                mma3(part[i], ah, al, bf);
             }
         }
+#pragma unroll
+        for (int i = 0; i < MT; ++i)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) acc[i][j] += part[i][j];
     }
 
     // ---- epilogue: D fragments -> sub_s[pol][pixel], then a3 + a4 + a5 ---------------------------

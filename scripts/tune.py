@@ -47,7 +47,7 @@ def main():
     print(json.dumps({"config": args.config, **kw, "stats": st}), flush=True)
     for kernel, env in (("gridder", "IDG_GRIDDER_VARIANT"), ("degridder", "IDG_DEGRIDDER_VARIANT")):
         for name in idg.idg.kernel_variants(kernel):
-            if not name.startswith(f"{kernel}<{ns},"):
+            if f"<{ns}," not in name:
                 continue
             if args.only and args.only not in name:
                 continue
