@@ -410,15 +410,15 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 #define TG(NS, W, MT, MB) \
     {NS, 8, kTensor, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB>}
 const Variant kTcGridder[] = {
-    TG(24, 6, 6, 2), TG(24, 12, 3, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
-    TG(32, 8, 8, 2), TG(32, 16, 4, 1), TG(32, 4, 16, 3), TG(32, 16, 4, 2),
+    TG(24, 12, 3, 2), TG(24, 6, 6, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
+    TG(32, 16, 4, 2), TG(32, 8, 8, 2), TG(32, 16, 4, 1), TG(32, 4, 16, 3),
     TG(16, 4, 4, 4), TG(16, 8, 2, 3), TG(16, 16, 1, 2),
 };
 #undef TG
 #define TD(NS, W, MT, MB) \
     {NS, 0, kTensor, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>}
 const Variant kTcDegridder[] = {
-    TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 2, 3), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
+    TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
     TD(32, 8, 4, 2), TD(32, 4, 4, 3), TD(32, 8, 8, 1), TD(32, 16, 2, 1),
     TD(16, 8, 4, 2), TD(16, 4, 4, 4), TD(16, 8, 2, 3),
 };
