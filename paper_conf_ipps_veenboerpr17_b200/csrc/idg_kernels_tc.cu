@@ -33,11 +33,41 @@ using dev::ItemSetup;
 
 __device__ __forceinline__ uint32_t h2_bits(__half2 h) { return *reinterpret_cast<uint32_t *>(&h); }
 
+// Packed f32x2 helpers (sm_100: FFMA2 / FMUL2 / FADD2 execute two fp32 lanes per issue slot).
+using f2p = uint64_t;
+__device__ __forceinline__ f2p pk(float lo, float hi) {
+    f2p r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+    return r;
+}
+__device__ __forceinline__ f2p dup(float v) { return pk(v, v); }
+__device__ __forceinline__ float2 unpk(f2p v) {
+    float2 r;
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(r.x), "=f"(r.y) : "l"(v));
+    return r;
+}
+__device__ __forceinline__ f2p fma2(f2p a, f2p b, f2p c) {
+    f2p r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+    return r;
+}
+__device__ __forceinline__ f2p mul2(f2p a, f2p b) {
+    f2p r;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ f2p sub2(f2p a, f2p b) {
+    f2p r;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+
 // (x, y) -> f16x2 hi = rn(x, y) and lo = rn(x - hi, y - hi): x = hi + lo to ~22 significant bits.
 __device__ __forceinline__ void split2(float x, float y, uint32_t &hi, uint32_t &lo) {
     const __half2 h = __floats2half2_rn(x, y);
     const float2 hf = __half22float2(h);
-    const __half2 l = __floats2half2_rn(x - hf.x, y - hf.y);
+    const float2 d = unpk(sub2(pk(x, y), pk(hf.x, hf.y)));  // one FADD2 for both residuals
+    const __half2 l = __floats2half2_rn(d.x, d.y);
     hi = h2_bits(h);
     lo = h2_bits(l);
 }
@@ -91,7 +121,7 @@ constexpr int kTcBatchKB = 64;  // k-blocks per shared-memory batch (512 visibil
 
 inline size_t gridder_tc_smem_bytes(int NS, int max_channels) {
     const size_t kbb = kTcBatchKB;
-    const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + kbb * 4 * 8 /*df*/ +
+    const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + kbb * 4 * 16 /*df*/ +
                         (kbb + 1) * 32 /*coef*/ + size_t(max_channels) * 4;
     const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2);
     return std::max(main, epi) + 16;
@@ -108,7 +138,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
     extern __shared__ __align__(16) unsigned char smem[];
     float4 *raw_s = reinterpret_cast<float4 *>(smem);                // [VB][2]
     uint4 *frag_s = reinterpret_cast<uint4 *>(raw_s + 2 * VB);       // [KBB][32]
-    float2 *dfk_s = reinterpret_cast<float2 *>(frag_s + KBB * 32);   // [KBB][4]
+    float4 *dfk_s = reinterpret_cast<float4 *>(frag_s + KBB * 32);   // [KBB][4] (df_q, df_q, df_q4, df_q4)
     float4 *coef_s = reinterpret_cast<float4 *>(dfk_s + KBB * 4);    // [KBB+1][2]
     float *df_s = reinterpret_cast<float *>(coef_s + 2 * (KBB + 1)); // [nc]
     __shared__ float red_s[WARPS];
@@ -125,17 +155,23 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
     for (int c = threadIdx.x; c < nc; c += NT)
         df_s[c] = float((a.frequencies[md.channel_begin + c] / kSpeedOfLight) - s.f_ref);
 
-    float pl[MT][2], pm[MT][2], pn[MT][2], acc[MT][4];
+    // (l, m, n) of the thread's two rows (pixels g and g+8 of each m-tile), packed as f32x2 pairs
+    f2p pl[MT], pm[MT], pn[MT];
+    float acc[MT][4];
 #pragma unroll
     for (int i = 0; i < MT; ++i) {
+        float l2[2], m2[2], n2[2];
 #pragma unroll
         for (int r = 0; r < 2; ++r) {
             const int pix = (warp * MT + i) * 16 + g + 8 * r;
             const int x = pix % NS, y = pix / NS;
-            pl[i][r] = float(x - h) * a.cell_l;
-            pm[i][r] = float(y - h) * a.cell_l;
-            pn[i][r] = dev::w_term_n(pl[i][r], pm[i][r]);
+            l2[r] = float(x - h) * a.cell_l;
+            m2[r] = float(y - h) * a.cell_l;
+            n2[r] = dev::w_term_n(l2[r], m2[r]);
         }
+        pl[i] = pk(l2[0], l2[1]);
+        pm[i] = pk(m2[0], m2[1]);
+        pn[i] = pk(n2[0], n2[1]);
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
     }
@@ -169,7 +205,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
         for (int i = threadIdx.x; i < (kb1 - kb0) * 4; i += NT) {
             const int kb = kb0 + (i >> 2);
             const int c = (kb % kpt) * 8 + (i & 3);
-            dfk_s[i] = make_float2(df_s[c], df_s[c + 4]);
+            dfk_s[i] = make_float4(df_s[c], df_s[c], df_s[c + 4], df_s[c + 4]);
         }
         __syncthreads();
         // (4) f16 range: power-of-two scale from the batch maximum; never increase the running scale
@@ -210,34 +246,35 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
         for (int i = 0; i < MT; ++i)
 #pragma unroll
             for (int j = 0; j < 4; ++j) part[i][j] = 0.0f;
-        int cur_t = -1;
-        float Bv[MT][2], Qv[MT][2];
-        for (int kb = kb0; kb < kb1; ++kb) {
-            const int t = kb / kpt;
-            if (t != cur_t) {
-                cur_t = t;
-                const float4 cB = coef_s[2 * (t - t_first)], cQ = coef_s[2 * (t - t_first) + 1];
-#pragma unroll
-                for (int i = 0; i < MT; ++i)
-#pragma unroll
-                    for (int r = 0; r < 2; ++r) {
-                        Bv[i][r] = fmaf(cB.x, pl[i][r], fmaf(cB.y, pm[i][r], cB.z * pn[i][r]));
-                        Qv[i][r] = fmaf(cQ.x, pl[i][r], fmaf(cQ.y, pm[i][r], cQ.z * pn[i][r]));
-                    }
-            }
-            const uint4 bf = frag_s[(kb - kb0) * 32 + lane];
-            const float2 df = dfk_s[(kb - kb0) * 4 + q];
+        for (int t = t_first; t <= t_last; ++t) {
+            // B_t, Q_t of both rows of every tile (packed pairs), once per timestep
+            const float4 cB = coef_s[2 * (t - t_first)], cQ = coef_s[2 * (t - t_first) + 1];
+            f2p Bv[MT], Qv[MT];
 #pragma unroll
             for (int i = 0; i < MT; ++i) {
-                float sn[4], cs[4];
-                __sincosf(fmaf(df.x, Qv[i][0], Bv[i][0]), &sn[0], &cs[0]);  // row g,   slot q
-                __sincosf(fmaf(df.x, Qv[i][1], Bv[i][1]), &sn[1], &cs[1]);  // row g+8, slot q
-                __sincosf(fmaf(df.y, Qv[i][0], Bv[i][0]), &sn[2], &cs[2]);  // row g,   slot q+4
-                __sincosf(fmaf(df.y, Qv[i][1], Bv[i][1]), &sn[3], &cs[3]);  // row g+8, slot q+4
-                uint32_t ah[4], al[4];
+                Bv[i] = fma2(dup(cB.x), pl[i], fma2(dup(cB.y), pm[i], mul2(dup(cB.z), pn[i])));
+                Qv[i] = fma2(dup(cQ.x), pl[i], fma2(dup(cQ.y), pm[i], mul2(dup(cQ.z), pn[i])));
+            }
+            const int k_begin = max(kb0, t * kpt), k_end = min(kb1, (t + 1) * kpt);
+#pragma unroll 1
+            for (int kb = k_begin; kb < k_end; ++kb) {
+                const uint4 bf = frag_s[(kb - kb0) * 32 + lane];
+                const float4 df = dfk_s[(kb - kb0) * 4 + q];
+                const f2p dq = pk(df.x, df.y), dq4 = pk(df.z, df.w);
 #pragma unroll
-                for (int j = 0; j < 4; ++j) split2(cs[j], sn[j], ah[j], al[j]);
-                mma3(part[i], ah, al, bf);
+                for (int i = 0; i < MT; ++i) {
+                    const float2 ph0 = unpk(fma2(dq, Qv[i], Bv[i]));   // (row g, row g+8) at slot q
+                    const float2 ph1 = unpk(fma2(dq4, Qv[i], Bv[i]));  // (row g, row g+8) at slot q+4
+                    float sn[4], cs[4];
+                    __sincosf(ph0.x, &sn[0], &cs[0]);
+                    __sincosf(ph0.y, &sn[1], &cs[1]);
+                    __sincosf(ph1.x, &sn[2], &cs[2]);
+                    __sincosf(ph1.y, &sn[3], &cs[3]);
+                    uint32_t ah[4], al[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) split2(cs[j], sn[j], ah[j], al[j]);
+                    mma3(part[i], ah, al, bf);
+                }
             }
         }
 #pragma unroll
@@ -268,7 +305,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
 // ------------------------------------------------------------------------------------------------
 inline size_t degridder_tc_smem_bytes(int NS) {
     const size_t npix = size_t(NS) * NS;
-    return npix * 64 /*sub+tmp | frag*/ + npix * 16 /*lmn*/ + 16;
+    return npix * 64 /*sub+tmp | frag*/ + npix * 4 * 8 / 2 /*lmn slot pairs: 32 B per 2 pixels*/ + 16;
 }
 
 template <int NS, int WARPS, int MT, int MINB>
@@ -283,7 +320,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     float2 *sub_s = reinterpret_cast<float2 *>(smem);                     // [4][NS][NS]
     float2 *tmp_s = sub_s + 4 * NPIX;                                     // [4][NS][NS]
     uint4 *frag_s = reinterpret_cast<uint4 *>(smem);                      // [NKB][32] (after prologue)
-    float4 *lmn_s = reinterpret_cast<float4 *>(smem + size_t(NPIX) * 64); // [NPIX]
+    float4 *lmn_s = reinterpret_cast<float4 *>(smem + size_t(NPIX) * 64); // [NKB][4][2] slot pairs
     __shared__ float red_s[WARPS];
     __shared__ float2 tw[NS];
 
@@ -305,7 +342,13 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
             for (int p = 0; p < 4; ++p) mx = fmaxf(mx, fmaxf(fabsf(rr[i][p].x), fabsf(rr[i][p].y)));
             const int y = pix / NS, x = pix - y * NS;
             const float l = float(x - h) * a.cell_l, m = float(y - h) * a.cell_l;
-            lmn_s[pix] = make_float4(l, m, dev::w_term_n(l, m), 0.0f);
+            // slot pair (q, q+4) of k-block kb: {l_q, l_q4, m_q, m_q4}, {n_q, n_q4, 0, 0}
+            const int kb = pix >> 3, slot = pix & 7, half = slot >> 2;
+            float *rec = reinterpret_cast<float *>(lmn_s + (kb * 4 + (slot & 3)) * 2);
+            rec[half] = l;
+            rec[2 + half] = m;
+            rec[4 + half] = dev::w_term_n(l, m);
+            rec[6 + half] = 0.0f;
         }
     }
     const float scale = pow2_scale(block_max<WARPS>(mx, red_s));  // barriers: tmp_s reads are done
@@ -337,36 +380,44 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
                    int64_t(md.channel_begin) * 4;
     for (int tile0 = warp * MT; tile0 < ntiles; tile0 += WARPS * MT) {
-        float cu[MT][2], cv[MT][2], cw[MT][2], acc[MT][4];
+        f2p cu[MT][2], cv[MT][2], cw[MT][2];  // (coefficient, coefficient) pairs of rows g and g+8
+        float acc[MT][4];
 #pragma unroll
         for (int i = 0; i < MT; ++i) {
 #pragma unroll
             for (int r = 0; r < 2; ++r) {
                 const int v = (tile0 + i) * 16 + g + 8 * r;
-                cu[i][r] = cv[i][r] = cw[i][r] = 0.0f;
+                float fu = 0.0f, fv = 0.0f, fw = 0.0f;
                 if (v < nvis) {
                     const int t = v / nc, c = v - t * nc;
                     const float *p = a.uvw + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset + t) * 3;
                     const double f = a.frequencies[md.channel_begin + c] / kSpeedOfLight;
-                    cu[i][r] = float(dev::kTwoPi * (double(p[0]) * f - s.u0));
-                    cv[i][r] = float(dev::kTwoPi * (double(p[1]) * f - s.v0));
-                    cw[i][r] = float(dev::kTwoPi * (double(p[2]) * f - s.w0));
+                    fu = float(dev::kTwoPi * (double(p[0]) * f - s.u0));
+                    fv = float(dev::kTwoPi * (double(p[1]) * f - s.v0));
+                    fw = float(dev::kTwoPi * (double(p[2]) * f - s.w0));
                 }
+                cu[i][r] = dup(fu);
+                cv[i][r] = dup(fv);
+                cw[i][r] = dup(fw);
             }
 #pragma unroll
             for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
         }
-#pragma unroll 2
+#pragma unroll 1
         for (int kb = 0; kb < NKB; ++kb) {
             const uint4 bf = frag_s[kb * 32 + lane];
-            const float4 x0 = lmn_s[kb * 8 + q], x1 = lmn_s[kb * 8 + q + 4];
+            const float4 lm = lmn_s[(kb * 4 + q) * 2], nn = lmn_s[(kb * 4 + q) * 2 + 1];
+            const f2p l2 = pk(lm.x, lm.y), m2 = pk(lm.z, lm.w), n2 = pk(nn.x, nn.y);
 #pragma unroll
             for (int i = 0; i < MT; ++i) {
+                // phases of (row, slot q) and (row, slot q+4) in one FFMA2 chain per row
+                const float2 p0 = unpk(fma2(cu[i][0], l2, fma2(cv[i][0], m2, mul2(cw[i][0], n2))));
+                const float2 p1 = unpk(fma2(cu[i][1], l2, fma2(cv[i][1], m2, mul2(cw[i][1], n2))));
                 float sn[4], cs[4];
-                __sincosf(fmaf(cu[i][0], x0.x, fmaf(cv[i][0], x0.y, cw[i][0] * x0.z)), &sn[0], &cs[0]);
-                __sincosf(fmaf(cu[i][1], x0.x, fmaf(cv[i][1], x0.y, cw[i][1] * x0.z)), &sn[1], &cs[1]);
-                __sincosf(fmaf(cu[i][0], x1.x, fmaf(cv[i][0], x1.y, cw[i][0] * x1.z)), &sn[2], &cs[2]);
-                __sincosf(fmaf(cu[i][1], x1.x, fmaf(cv[i][1], x1.y, cw[i][1] * x1.z)), &sn[3], &cs[3]);
+                __sincosf(p0.x, &sn[0], &cs[0]);  // row g,   slot q
+                __sincosf(p1.x, &sn[1], &cs[1]);  // row g+8, slot q
+                __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
+                __sincosf(p1.y, &sn[3], &cs[3]);  // row g+8, slot q+4
                 uint32_t ah[4], al[4];
 #pragma unroll
                 for (int j = 0; j < 4; ++j) split2(cs[j], sn[j], ah[j], al[j]);
@@ -411,14 +462,16 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
     {NS, 8, kTensor, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB>}
 const Variant kTcGridder[] = {
     TG(24, 12, 3, 2), TG(24, 6, 6, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
-    TG(32, 16, 4, 2), TG(32, 8, 8, 2), TG(32, 16, 4, 1), TG(32, 4, 16, 3),
+    TG(24, 6, 6, 3), TG(24, 9, 4, 3), TG(24, 4, 9, 4),
+    TG(32, 16, 4, 2), TG(32, 8, 8, 2), TG(32, 16, 4, 1), TG(32, 4, 16, 3), TG(32, 8, 8, 3),
     TG(16, 4, 4, 4), TG(16, 8, 2, 3), TG(16, 16, 1, 2),
 };
 #undef TG
 #define TD(NS, W, MT, MB) \
     {NS, 0, kTensor, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>}
 const Variant kTcDegridder[] = {
-    TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
+    TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1), TD(24, 8, 2, 4),
+    TD(24, 4, 2, 6),
     TD(32, 8, 4, 2), TD(32, 4, 4, 3), TD(32, 8, 8, 1), TD(32, 16, 2, 1),
     TD(16, 8, 4, 2), TD(16, 4, 4, 4), TD(16, 8, 2, 3),
 };
