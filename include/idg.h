@@ -136,7 +136,8 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
  * idg_rho_benchmark -- the paper's FMA:sincos throughput benchmark (Fig. 12) on the
  * current device: every sincos evaluation is followed by rho-1 FMAs plus the one FMA that forms its
  * argument (rho FMAs per sincos).  ops = 2 per FMA + 1 per sin + 1 per cos (op definition).
- *   rho in {1,2,3,4,6,8,12,16,17,20,24,32,48,64};  iterations >= 1 (work per thread);  ops_per_second receives the measured
+ *   rho in {0,1,2,3,4,6,8,12,16,17,20,24,32,48,64}; rho = 0 measures sincos alone (2 ops each: the
+ *   XU/MUFU bound of the tensor-core kernels, whose multiply-adds run on the tensor cores);  iterations >= 1 (work per thread);  ops_per_second receives the measured
  *   throughput (synchronous: the call waits for the kernel; timed with CUDA events on `stream`).
  */
 idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream,
@@ -159,7 +160,9 @@ idg_status idg_profiling_read(idg_kernel_time *dst, int32_t capacity, int32_t *n
 
 /* Diagnostics: newline-separated names of the compiled launch-shape variants of the gridder
  * (which = 0) or degridder (which = 1).  Setting the environment variable IDG_GRIDDER_VARIANT /
- * IDG_DEGRIDDER_VARIANT to one of these names before a call overrides the default (tuning only). */
+ * IDG_DEGRIDDER_VARIANT to one of these names before a call overrides the default (tuning only);
+ * the values "tc" (direct tensor-core kernel) and "simt" (CUDA-core kernel, the paper's structure)
+ * select a kernel family.  The default is the fastest eligible tensor-core variant. */
 const char *idg_kernel_variants(int32_t which);
 
 /* Number of kernel launches issued by this library in the calling process so far. */

@@ -63,6 +63,8 @@ struct idg_plan {
     int64_t nr_vis_assigned = 0, nr_vis_dropped = 0, nr_pairs = 0;
     int32_t max_channels_in_item = 0;
     int32_t channel_gcd = 1;
+    int32_t channels_uniform = 0;
+    float channel_step = 0.0f;
     mutable std::mutex mu;
     mutable std::map<int, DeviceCopy> device;
 
@@ -197,6 +199,8 @@ idg::KernelArgs make_args(const idg_plan *plan, const DeviceCopy *dc, const floa
     a.grid = static_cast<float2 *>(d_grid);
     a.max_channels_in_item = plan->max_channels_in_item;
     a.channel_gcd = plan->channel_gcd;
+    a.channels_uniform = plan->channels_uniform;
+    a.channel_step = plan->channel_step;
     return a;
 }
 
@@ -282,6 +286,15 @@ idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, i
             g = std::gcd(g, nc);
         }
         plan->channel_gcd = g == 0 ? 1 : g;
+        // uniform channel spacing (enables the phasor recurrence over channels in the gridder)
+        if (nr_channels >= 2) {
+            const double d0 = frequencies[1] - frequencies[0];
+            bool uni = d0 != 0.0;
+            for (int32_t c = 1; c + 1 < nr_channels && uni; ++c)
+                uni = std::fabs((frequencies[c + 1] - frequencies[c]) - d0) <= 1e-9 * std::fabs(frequencies[0]);
+            plan->channels_uniform = uni ? 1 : 0;
+            plan->channel_step = float(d0 / idg::kSpeedOfLight);
+        }
         plan->order.resize(plan->items.size());
         std::iota(plan->order.begin(), plan->order.end(), 0);
         std::stable_sort(plan->order.begin(), plan->order.end(), [&](int32_t a, int32_t b) {
@@ -379,11 +392,11 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
 
 idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
                              double *seconds) {
-    static const int kSupported[] = {1, 2, 3, 4, 6, 8, 12, 16, 17, 20, 24, 32, 48, 64};
+    static const int kSupported[] = {0, 1, 2, 3, 4, 6, 8, 12, 16, 17, 20, 24, 32, 48, 64};
     if (std::find(std::begin(kSupported), std::end(kSupported), rho) == std::end(kSupported) ||
         iterations < 1 || !ops_per_second)
         return fail(IDG_ERR_INVALID_ARG,
-                    "rho in {1,2,3,4,6,8,12,16,17,20,24,32,48,64}, iterations >= 1, ops_per_second != NULL");
+                    "rho in {0,1,2,3,4,6,8,12,16,17,20,24,32,48,64}, iterations >= 1, ops_per_second != NULL");
     const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
     float *d_out = nullptr;
     cudaError_t e = cudaMalloc(&d_out, sizeof(float) * 148 * 64 * 256);

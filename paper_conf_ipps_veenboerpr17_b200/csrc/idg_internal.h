@@ -46,6 +46,8 @@ struct KernelArgs {
     float2 *grid;                // [4][N][N]       (const for degridding)
     int32_t max_channels_in_item;
     int32_t channel_gcd;         // gcd of all items' channel counts
+    int32_t channels_uniform;    // 1 if nu_{c+1} - nu_c is the same for all c (to 1e-9 relative)
+    float channel_step;          // (nu_{c+1} - nu_c) / c  [1/m], valid when channels_uniform
 };
 
 using Launcher = cudaError_t (*)(const KernelArgs &, cudaStream_t);
@@ -54,6 +56,7 @@ struct Variant {
     int ns;            // subgrid size
     int v;             // channels per thread (SIMT degridder) / channel multiple (tensor gridder); 0 = any
     int kind;          // kSimt | kTensor
+    int needs_uniform; // 1: requires uniformly spaced channels (phasor recurrence over channels)
     const char *name;
     Launcher fn;
 };

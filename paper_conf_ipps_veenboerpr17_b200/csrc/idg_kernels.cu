@@ -300,14 +300,14 @@ cudaError_t launch_degridder_t(const KernelArgs &a, cudaStream_t st) {
 
 // SIMT launch-shape variants (first entry per (NS, V) is the SIMT default; tuned with scripts/tune.py).
 // v = channels per thread for the degridder (every item's channel count must be a multiple of v).
-#define GV(NS, P, MB) {NS, 0, kSimt, "gridder<" #NS ",P" #P ",minB" #MB ">", launch_gridder_t<NS, P, MB>}
+#define GV(NS, P, MB) {NS, 0, kSimt, 0, "gridder<" #NS ",P" #P ",minB" #MB ">", launch_gridder_t<NS, P, MB>}
 const Variant kGridderVariants[] = {
     GV(24, 6, 4), GV(24, 6, 5), GV(24, 6, 6), GV(24, 3, 3), GV(24, 3, 4), GV(24, 2, 4), GV(24, 9, 3),
     GV(32, 4, 2), GV(32, 8, 3), GV(32, 8, 4), GV(32, 4, 3), GV(32, 16, 4),
     GV(16, 4, 4), GV(16, 4, 6), GV(16, 2, 4), GV(16, 8, 6),
 };
 #undef GV
-#define DV(NS, V, NT, MB) {NS, V, kSimt, "degridder<" #NS ",V" #V ",T" #NT ",minB" #MB ">", launch_degridder_t<NS, V, NT, MB>}
+#define DV(NS, V, NT, MB) {NS, V, kSimt, 0, "degridder<" #NS ",V" #V ",T" #NT ",minB" #MB ">", launch_degridder_t<NS, V, NT, MB>}
 #define DV_ALL(NS) DV(NS, 8, 128, 4), DV(NS, 8, 128, 3), DV(NS, 8, 256, 1), DV(NS, 8, 256, 2), \
     DV(NS, 8, 64, 6), DV(NS, 8, 64, 8), DV(NS, 4, 128, 4), DV(NS, 4, 256, 3), DV(NS, 4, 128, 6), \
     DV(NS, 2, 128, 6), DV(NS, 1, 128, 6)
@@ -315,30 +315,32 @@ const Variant kDegridderVariants[] = {DV_ALL(24), DV_ALL(32), DV_ALL(16)};
 #undef DV_ALL
 #undef DV
 
-bool eligible(const Variant &var, int ns, int channel_gcd) {
-    if (var.ns != ns) return false;
-    if (var.kind == kTensor) return var.v == 0 || channel_gcd % var.v == 0;
-    return var.v == 0 || channel_gcd % var.v == 0;
+bool eligible(const Variant &var, const KernelArgs &a) {
+    if (var.ns != a.subgrid_size) return false;
+    if (var.needs_uniform && !a.channels_uniform) return false;
+    return var.v == 0 || a.channel_gcd % var.v == 0;
 }
 
 // Variant choice.  Default: the first eligible tensor-core variant, else the first eligible SIMT
 // variant (for the SIMT degridder: the one with the largest channels-per-thread).  The environment
 // variable `env` (IDG_GRIDDER_VARIANT / IDG_DEGRIDDER_VARIANT) may name any eligible variant (tuning).
-const Variant *pick(const Variant *simt, int nsimt, const Variant *tc, int ntc, int ns, int channel_gcd,
+const Variant *pick(const Variant *simt, int nsimt, const Variant *tc, int ntc, const KernelArgs &a,
                     const char *env) {
     const char *want = std::getenv(env);
     if (want && *want) {
         for (int i = 0; i < ntc; ++i)
-            if (eligible(tc[i], ns, channel_gcd) && std::strcmp(want, tc[i].name) == 0) return &tc[i];
+            if (eligible(tc[i], a) && std::strcmp(want, tc[i].name) == 0) return &tc[i];
         for (int i = 0; i < nsimt; ++i)
-            if (eligible(simt[i], ns, channel_gcd) && std::strcmp(want, simt[i].name) == 0) return &simt[i];
+            if (eligible(simt[i], a) && std::strcmp(want, simt[i].name) == 0) return &simt[i];
     }
+    // "tc": the direct tensor-core kernel (no channel recurrence); "simt": the CUDA-core kernel
+    const bool tc_direct = want && std::strcmp(want, "tc") == 0;
     if (!(want && std::strcmp(want, "simt") == 0))
         for (int i = 0; i < ntc; ++i)
-            if (eligible(tc[i], ns, channel_gcd)) return &tc[i];
+            if (eligible(tc[i], a) && !(tc_direct && tc[i].needs_uniform)) return &tc[i];
     const Variant *best = nullptr;
     for (int i = 0; i < nsimt; ++i)
-        if (eligible(simt[i], ns, channel_gcd) && (!best || simt[i].v > best->v)) best = &simt[i];
+        if (eligible(simt[i], a) && (!best || simt[i].v > best->v)) best = &simt[i];
     return best;
 }
 
@@ -348,8 +350,8 @@ cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
     int ntc = 0;
     const Variant *tc = tc_gridder_variants(&ntc);
-    const Variant *var = pick(kGridderVariants, int(std::size(kGridderVariants)), tc, ntc, a.subgrid_size,
-                              a.channel_gcd, "IDG_GRIDDER_VARIANT");
+    const Variant *var = pick(kGridderVariants, int(std::size(kGridderVariants)), tc, ntc, a,
+                              "IDG_GRIDDER_VARIANT");
     return var ? var->fn(a, s) : cudaErrorInvalidValue;
 }
 
@@ -357,8 +359,8 @@ cudaError_t launch_degridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
     int ntc = 0;
     const Variant *tc = tc_degridder_variants(&ntc);
-    const Variant *var = pick(kDegridderVariants, int(std::size(kDegridderVariants)), tc, ntc, a.subgrid_size,
-                              a.channel_gcd, "IDG_DEGRIDDER_VARIANT");
+    const Variant *var = pick(kDegridderVariants, int(std::size(kDegridderVariants)), tc, ntc, a,
+                              "IDG_DEGRIDDER_VARIANT");
     return var ? var->fn(a, s) : cudaErrorInvalidValue;
 }
 

@@ -56,6 +56,30 @@ __global__ void __launch_bounds__(kRhoThreads) rho_kernel(float *out, int iterat
     out[tid] = sum;
 }
 
+// rho = 0: sincos throughput alone (the XU/MUFU bound of the tensor-core kernels).  Eight independent
+// chains per thread; the next argument is cos * 0.5 + sin (one FMA that is not counted as an op).
+template <>
+__global__ void __launch_bounds__(kRhoThreads) rho_kernel<0>(float *out, int iterations) {
+    constexpr int U = 8;
+    const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+    float x[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) x[k] = 1e-3f * float(tid & 255) + float(k);
+#pragma unroll 1
+    for (int i = 0; i < iterations; ++i) {
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            float sn, cs;
+            __sincosf(x[k], &sn, &cs);
+            x[k] = fmaf(cs, 0.5f, sn);
+        }
+    }
+    float sum = 0.0f;
+#pragma unroll
+    for (int k = 0; k < U; ++k) sum += x[k];
+    out[tid] = sum;
+}
+
 template <int RHO>
 cudaError_t run(int iterations, float *out, cudaStream_t s, int *blocks) {
     int per_sm = 0, dev = 0;
@@ -74,8 +98,9 @@ cudaError_t run(int iterations, float *out, cudaStream_t s, int *blocks) {
 cudaError_t launch_rho_benchmark(int rho, int iterations, float *d_out, cudaStream_t s, int *blocks,
                                  int *threads, int *units_per_thread) {
     *threads = kRhoThreads;
-    *units_per_thread = kRhoUnits;
+    *units_per_thread = rho == 0 ? 8 : kRhoUnits;
     switch (rho) {
+        case 0: return run<0>(iterations, d_out, s, blocks);
 #define IDG_RHO_CASE(R) \
     case R: return run<R>(iterations, d_out, s, blocks);
         IDG_RHO_CASE(1) IDG_RHO_CASE(2) IDG_RHO_CASE(3) IDG_RHO_CASE(4) IDG_RHO_CASE(6)

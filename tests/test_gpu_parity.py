@@ -69,12 +69,13 @@ CASES = [
 ]
 
 
-@pytest.fixture(params=["default", "simt"])
+@pytest.fixture(params=["default", "tc", "simt"])
 def kind(request, monkeypatch):
-    """default = tensor-core kernels where eligible; simt = the paper-structured CUDA-core kernels."""
-    if request.param == "simt":
-        monkeypatch.setenv("IDG_GRIDDER_VARIANT", "simt")
-        monkeypatch.setenv("IDG_DEGRIDDER_VARIANT", "simt")
+    """default = fastest tensor-core kernels (channel recurrence where channels are uniform);
+    tc = direct tensor-core kernels; simt = the paper-structured CUDA-core kernels."""
+    if request.param != "default":
+        monkeypatch.setenv("IDG_GRIDDER_VARIANT", request.param)
+        monkeypatch.setenv("IDG_DEGRIDDER_VARIANT", request.param)
     return request.param
 
 
