@@ -161,8 +161,9 @@ idg_status idg_profiling_read(idg_kernel_time *dst, int32_t capacity, int32_t *n
 /* Diagnostics: newline-separated names of the compiled launch-shape variants of the gridder
  * (which = 0) or degridder (which = 1).  Setting the environment variable IDG_GRIDDER_VARIANT /
  * IDG_DEGRIDDER_VARIANT to one of these names before a call overrides the default (tuning only);
- * the values "tc" (direct tensor-core kernel) and "simt" (CUDA-core kernel, the paper's structure)
- * select a kernel family.  The default is the fastest eligible tensor-core variant. */
+ * a name prefix ending in '*' selects the first eligible match; the values "tc" (direct tensor-core
+ * kernel) and "simt" (CUDA-core kernel, the paper's structure) select a kernel family.  The default
+ * is the fastest eligible tensor-core variant. */
 const char *idg_kernel_variants(int32_t which);
 
 /* Number of kernel launches issued by this library in the calling process so far. */

@@ -61,8 +61,10 @@ struct Variant {
     Launcher fn;
 };
 // Tensor-core variants (idg_kernels_tc.cu); the first eligible one is the default.
-const Variant *tc_gridder_variants(int *n);
+const Variant *tc_gridder_variants(int *n);     // split-f16 mma (idg_kernels_tc.cu)
 const Variant *tc_degridder_variants(int *n);
+const Variant *tf32_gridder_variants(int *n);   // split-tf32 mma (idg_kernels_tf32.cu)
+const Variant *tf32_degridder_variants(int *n);
 
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s);
 cudaError_t launch_degridder(const KernelArgs &a, cudaStream_t s);

@@ -27,6 +27,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <vector>
 
 #include "idg_device.cuh"
 #include "idg_internal.h"
@@ -324,58 +325,81 @@ bool eligible(const Variant &var, const KernelArgs &a) {
 // Variant choice.  Default: the first eligible tensor-core variant, else the first eligible SIMT
 // variant (for the SIMT degridder: the one with the largest channels-per-thread).  The environment
 // variable `env` (IDG_GRIDDER_VARIANT / IDG_DEGRIDDER_VARIANT) may name any eligible variant (tuning).
-const Variant *pick(const Variant *simt, int nsimt, const Variant *tc, int ntc, const KernelArgs &a,
+const Variant *pick(const Variant *simt, int nsimt, const std::vector<const Variant *> &tc, const KernelArgs &a,
                     const char *env) {
     const char *want = std::getenv(env);
     if (want && *want) {
-        for (int i = 0; i < ntc; ++i)
-            if (eligible(tc[i], a) && std::strcmp(want, tc[i].name) == 0) return &tc[i];
+        // exact name, or a prefix ending in '*' (first eligible match)
+        const size_t len = std::strlen(want);
+        const bool prefix = want[len - 1] == '*';
+        auto match = [&](const char *name) {
+            return prefix ? std::strncmp(want, name, len - 1) == 0 : std::strcmp(want, name) == 0;
+        };
+        for (const Variant *v : tc)
+            if (eligible(*v, a) && match(v->name)) return v;
         for (int i = 0; i < nsimt; ++i)
-            if (eligible(simt[i], a) && std::strcmp(want, simt[i].name) == 0) return &simt[i];
+            if (eligible(simt[i], a) && match(simt[i].name)) return &simt[i];
     }
     // "tc": the direct tensor-core kernel (no channel recurrence); "simt": the CUDA-core kernel
     const bool tc_direct = want && std::strcmp(want, "tc") == 0;
     if (!(want && std::strcmp(want, "simt") == 0))
-        for (int i = 0; i < ntc; ++i)
-            if (eligible(tc[i], a) && !(tc_direct && tc[i].needs_uniform)) return &tc[i];
+        for (const Variant *v : tc)
+            if (eligible(*v, a) && !(tc_direct && v->needs_uniform)) return v;
     const Variant *best = nullptr;
     for (int i = 0; i < nsimt; ++i)
         if (eligible(simt[i], a) && (!best || simt[i].v > best->v)) best = &simt[i];
     return best;
 }
 
+// All tensor-core variants in default-preference order (measured on B200).
+const std::vector<const Variant *> &tensor_variants(int which) {
+    static const std::vector<const Variant *> lists[2] = {
+        [] {
+            std::vector<const Variant *> v;
+            int n = 0;
+            const Variant *t = tf32_gridder_variants(&n);
+            for (int i = 0; i < n; ++i) v.push_back(&t[i]);
+            t = tc_gridder_variants(&n);
+            for (int i = 0; i < n; ++i) v.push_back(&t[i]);
+            return v;
+        }(),
+        [] {
+            std::vector<const Variant *> v;
+            int n = 0;
+            const Variant *t = tf32_degridder_variants(&n);
+            for (int i = 0; i < n; ++i) v.push_back(&t[i]);
+            t = tc_degridder_variants(&n);
+            for (int i = 0; i < n; ++i) v.push_back(&t[i]);
+            return v;
+        }()};
+    return lists[which];
+}
+
 }  // namespace
 
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
-    int ntc = 0;
-    const Variant *tc = tc_gridder_variants(&ntc);
-    const Variant *var = pick(kGridderVariants, int(std::size(kGridderVariants)), tc, ntc, a,
+    const Variant *var = pick(kGridderVariants, int(std::size(kGridderVariants)), tensor_variants(0), a,
                               "IDG_GRIDDER_VARIANT");
     return var ? var->fn(a, s) : cudaErrorInvalidValue;
 }
 
 cudaError_t launch_degridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
-    int ntc = 0;
-    const Variant *tc = tc_degridder_variants(&ntc);
-    const Variant *var = pick(kDegridderVariants, int(std::size(kDegridderVariants)), tc, ntc, a,
+    const Variant *var = pick(kDegridderVariants, int(std::size(kDegridderVariants)), tensor_variants(1), a,
                               "IDG_DEGRIDDER_VARIANT");
     return var ? var->fn(a, s) : cudaErrorInvalidValue;
 }
 
 const char *variant_names(int which) {
-    static std::string g, d;
-    if (g.empty()) {
-        int n = 0;
-        const Variant *tc = tc_gridder_variants(&n);
-        for (int i = 0; i < n; ++i) g += std::string(tc[i].name) + "\n";
-        for (const Variant &v : kGridderVariants) g += std::string(v.name) + "\n";
-        tc = tc_degridder_variants(&n);
-        for (int i = 0; i < n; ++i) d += std::string(tc[i].name) + "\n";
-        for (const Variant &v : kDegridderVariants) d += std::string(v.name) + "\n";
+    static std::string names[2];
+    if (names[0].empty()) {
+        for (const Variant *v : tensor_variants(0)) names[0] += std::string(v->name) + "\n";
+        for (const Variant &v : kGridderVariants) names[0] += std::string(v.name) + "\n";
+        for (const Variant *v : tensor_variants(1)) names[1] += std::string(v->name) + "\n";
+        for (const Variant &v : kDegridderVariants) names[1] += std::string(v.name) + "\n";
     }
-    return which == 0 ? g.c_str() : d.c_str();
+    return names[which == 0 ? 0 : 1].c_str();
 }
 
 }  // namespace idg

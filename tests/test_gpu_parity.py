@@ -69,13 +69,23 @@ CASES = [
 ]
 
 
-@pytest.fixture(params=["default", "tc", "simt"])
+KINDS = {
+    "default": (None, None),                       # fastest tensor-core kernels (tf32 split, recurrence)
+    "tc": ("tc", "tc"),                            # direct tensor-core kernels (no channel recurrence)
+    "f16": ("gridder_tcr<*", "degridder_tc<*"),    # split-f16 tensor-core kernels
+    "f16direct": ("gridder_tc<*", "degridder_tc<*"),
+    "simt": ("simt", "simt"),                      # CUDA-core kernels (the paper's structure)
+}
+
+
+@pytest.fixture(params=list(KINDS))
 def kind(request, monkeypatch):
-    """default = fastest tensor-core kernels (channel recurrence where channels are uniform);
-    tc = direct tensor-core kernels; simt = the paper-structured CUDA-core kernels."""
-    if request.param != "default":
-        monkeypatch.setenv("IDG_GRIDDER_VARIANT", request.param)
-        monkeypatch.setenv("IDG_DEGRIDDER_VARIANT", request.param)
+    """Kernel family under test (the variant environment overrides of include/idg.h).  Families a
+    case is not eligible for (e.g. tensor-core gridders need C~ % 8 == 0) fall back to the default."""
+    g, d = KINDS[request.param]
+    if g:
+        monkeypatch.setenv("IDG_GRIDDER_VARIANT", g)
+        monkeypatch.setenv("IDG_DEGRIDDER_VARIANT", d)
     return request.param
 
 
