@@ -357,18 +357,18 @@ const std::vector<const Variant *> &tensor_variants(int which) {
         [] {
             std::vector<const Variant *> v;
             int n = 0;
-            const Variant *t = tf32_gridder_variants(&n);
+            const Variant *t = tc_gridder_variants(&n);
             for (int i = 0; i < n; ++i) v.push_back(&t[i]);
-            t = tc_gridder_variants(&n);
+            t = tf32_gridder_variants(&n);
             for (int i = 0; i < n; ++i) v.push_back(&t[i]);
             return v;
         }(),
         [] {
             std::vector<const Variant *> v;
             int n = 0;
-            const Variant *t = tf32_degridder_variants(&n);
+            const Variant *t = tc_degridder_variants(&n);
             for (int i = 0; i < n; ++i) v.push_back(&t[i]);
-            t = tc_degridder_variants(&n);
+            t = tf32_degridder_variants(&n);
             for (int i = 0; i < n; ++i) v.push_back(&t[i]);
             return v;
         }()};

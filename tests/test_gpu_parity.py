@@ -70,10 +70,10 @@ CASES = [
 
 
 KINDS = {
-    "default": (None, None),                       # fastest tensor-core kernels (tf32 split, recurrence)
+    "default": (None, None),                       # default tensor-core kernels (split-f16 mma)
     "tc": ("tc", "tc"),                            # direct tensor-core kernels (no channel recurrence)
-    "f16": ("gridder_tcr<*", "degridder_tc<*"),    # split-f16 tensor-core kernels
-    "f16direct": ("gridder_tc<*", "degridder_tc<*"),
+    "rec": ("gridder_tcr<*", "degridder_tc<*"),    # split-f16 gridder with the channel recurrence
+    "tf32": ("gridder_tf32*", "degridder_tf32*"),  # split-tf32 tensor-core kernels
     "simt": ("simt", "simt"),                      # CUDA-core kernels (the paper's structure)
 }
 
