@@ -102,7 +102,8 @@ idg_status idg_plan_metadata(const idg_plan *plan, idg_metadata *dst, int64_t n)
 idg_status idg_plan_stats(const idg_plan *plan, int64_t *nr_vis_assigned, int64_t *nr_vis_dropped,
                           int64_t *nr_pairs);
 
-/* Device workspace the grid/degrid calls need, in bytes (0 for the fused sm_100a kernels). */
+/* Device workspace idg_grid / idg_degrid need, in bytes (0: the fused sm_100a kernels keep every
+ * subgrid on chip).  The host-streamed calls need idg_host_workspace_size() instead. */
 idg_status idg_workspace_size(const idg_plan *plan, size_t *bytes);
 
 /*
@@ -131,6 +132,28 @@ idg_status idg_grid(const idg_plan *plan, const void *d_vis, const float *d_uvw,
 idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_uvw,
                       const void *d_aterms, const float *d_taper, void *d_vis, void *d_workspace,
                       size_t workspace_bytes, idg_stream stream);
+
+/*
+ * Host-streamed calls: the paper's asynchronous I/O (Fig. 7).  The visibilities live in
+ * HOST memory (page-locked for overlap, e.g. cudaHostAlloc / torch pin_memory) and stream through
+ * triple-buffered device staging buffers in work groups of contiguous baselines: uploads on an
+ * internal copy stream, kernels on `stream`, downloads on another internal copy stream, ordered with
+ * events, so transfers overlap the kernels.  Semantics are those of idg_grid / idg_degrid:
+ *   idg_grid_host    h_vis (read) -> d_grid (ACCUMULATED)
+ *   idg_degrid_host  d_grid -> h_vis (OVERWRITTEN, dropped visibilities = 0)
+ * d_workspace must hold idg_host_workspace_size() bytes (separate halves for the two directions, so a
+ * grid call's uploads can overlap a preceding degrid call).  Both calls are asynchronous on `stream`;
+ * h_vis must stay valid (and, for idg_grid_host, unmodified) until `stream` reaches the call's end.
+ * Calls on the same plan are serialised internally (the pipeline streams and events belong to the
+ * plan's device copy).
+ */
+idg_status idg_host_workspace_size(const idg_plan *plan, size_t *bytes);
+idg_status idg_grid_host(const idg_plan *plan, const void *h_vis, const float *d_uvw,
+                         const void *d_aterms, const float *d_taper, void *d_grid, void *d_workspace,
+                         size_t workspace_bytes, idg_stream stream);
+idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float *d_uvw,
+                           const void *d_aterms, const float *d_taper, void *h_vis, void *d_workspace,
+                           size_t workspace_bytes, idg_stream stream);
 
 /*
  * idg_rho_benchmark -- the paper's FMA:sincos throughput benchmark (Fig. 12) on the

@@ -6,6 +6,7 @@
 #include <cmath>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
 #include <map>
 #include <memory>
 #include <mutex>
@@ -41,11 +42,27 @@ std::atomic<bool> g_prof_enabled{false};
 std::vector<ProfileRecord> g_prof_pending;
 std::map<std::string, std::pair<int64_t, double>> g_prof_totals;
 
+constexpr int kStagingBuffers = 3;                  // triple buffering (Fig. 7)
+constexpr size_t kHostChunkBytes = size_t(128) << 20;  // visibilities per work group (host-streamed calls)
+
 struct DeviceCopy {
     idg_metadata *items = nullptr;
-    int32_t *order = nullptr;
+    int32_t *order = nullptr;      // launch order of the device-resident calls (largest work first)
+    int32_t *iota = nullptr;       // plan order (work groups of the host-streamed calls)
     int32_t *baselines = nullptr;
     double *frequencies = nullptr;
+    // host-streamed pipeline: one copy stream per direction + per-buffer events
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t ev_h2d[kStagingBuffers] = {}, ev_kernel_g[kStagingBuffers] = {};
+    cudaEvent_t ev_kernel_d[kStagingBuffers] = {}, ev_d2h[kStagingBuffers] = {};
+    std::mutex *pipeline_mu = nullptr;
+};
+
+// A work group of the host-streamed calls: baselines [b0, b1) (contiguous in host memory) and their
+// items [i0, i1) in plan order ("grouping m <= n work items into a work group").
+struct WorkGroup {
+    int32_t b0, b1;
+    int64_t i0, i1;
 };
 
 bool supported_subgrid(int32_t n) { return n == 16 || n == 24 || n == 32; }
@@ -62,6 +79,8 @@ struct idg_plan {
     std::vector<int32_t> order;      // launch order: largest T~ C~ first (tail balance)
     int64_t nr_vis_assigned = 0, nr_vis_dropped = 0, nr_pairs = 0;
     int32_t max_channels_in_item = 0;
+    std::vector<WorkGroup> groups;   // host-streamed work groups
+    size_t group_bytes = 0;          // largest work group's visibility bytes
     int32_t channel_gcd = 1;
     int32_t channels_uniform = 0;
     float channel_step = 0.0f;
@@ -75,6 +94,16 @@ struct idg_plan {
             cudaSetDevice(kv.first);
             cudaFree(kv.second.items);
             cudaFree(kv.second.order);
+            cudaFree(kv.second.iota);
+            if (kv.second.h2d) cudaStreamDestroy(kv.second.h2d);
+            if (kv.second.d2h) cudaStreamDestroy(kv.second.d2h);
+            for (int b = 0; b < kStagingBuffers; ++b) {
+                if (kv.second.ev_h2d[b]) cudaEventDestroy(kv.second.ev_h2d[b]);
+                if (kv.second.ev_kernel_g[b]) cudaEventDestroy(kv.second.ev_kernel_g[b]);
+                if (kv.second.ev_kernel_d[b]) cudaEventDestroy(kv.second.ev_kernel_d[b]);
+                if (kv.second.ev_d2h[b]) cudaEventDestroy(kv.second.ev_d2h[b]);
+            }
+            delete kv.second.pipeline_mu;
             cudaFree(kv.second.baselines);
             cudaFree(kv.second.frequencies);
             if (prev >= 0) cudaSetDevice(prev);
@@ -103,16 +132,31 @@ struct idg_plan {
         const size_t ni = std::max<size_t>(1, items.size());
         if ((e = cudaMalloc(&dc.items, ni * sizeof(idg_metadata))) != cudaSuccess ||
             (e = cudaMalloc(&dc.order, ni * sizeof(int32_t))) != cudaSuccess ||
+            (e = cudaMalloc(&dc.iota, ni * sizeof(int32_t))) != cudaSuccess ||
             (e = cudaMalloc(&dc.baselines, std::max<size_t>(2, baselines.size()) * 4)) != cudaSuccess ||
             (e = cudaMalloc(&dc.frequencies, frequencies.size() * 8)) != cudaSuccess) {
-            cudaFree(dc.items); cudaFree(dc.order); cudaFree(dc.baselines); cudaFree(dc.frequencies);
+            cudaFree(dc.items); cudaFree(dc.order); cudaFree(dc.iota); cudaFree(dc.baselines);
+            cudaFree(dc.frequencies);
             return e == cudaErrorMemoryAllocation ? fail(IDG_ERR_OUT_OF_MEMORY, "plan device copy")
                                                   : cuda_fail(e, "cudaMalloc(plan)");
         }
         if (!items.empty()) {
             cudaMemcpy(dc.items, items.data(), items.size() * sizeof(idg_metadata), cudaMemcpyHostToDevice);
             cudaMemcpy(dc.order, order.data(), order.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
+            std::vector<int32_t> iota(items.size());
+            std::iota(iota.begin(), iota.end(), 0);
+            cudaMemcpy(dc.iota, iota.data(), iota.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
         }
+        if ((e = cudaStreamCreateWithFlags(&dc.h2d, cudaStreamNonBlocking)) != cudaSuccess ||
+            (e = cudaStreamCreateWithFlags(&dc.d2h, cudaStreamNonBlocking)) != cudaSuccess)
+            return cuda_fail(e, "cudaStreamCreate(pipeline)");
+        for (int b = 0; b < kStagingBuffers; ++b) {
+            cudaEventCreateWithFlags(&dc.ev_h2d[b], cudaEventDisableTiming);
+            cudaEventCreateWithFlags(&dc.ev_kernel_g[b], cudaEventDisableTiming);
+            cudaEventCreateWithFlags(&dc.ev_kernel_d[b], cudaEventDisableTiming);
+            cudaEventCreateWithFlags(&dc.ev_d2h[b], cudaEventDisableTiming);
+        }
+        dc.pipeline_mu = new std::mutex();
         if (!baselines.empty())
             cudaMemcpy(dc.baselines, baselines.data(), baselines.size() * 4, cudaMemcpyHostToDevice);
         e = cudaMemcpy(dc.frequencies, frequencies.data(), frequencies.size() * 8, cudaMemcpyHostToDevice);
@@ -295,6 +339,21 @@ idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, i
             plan->channels_uniform = uni ? 1 : 0;
             plan->channel_step = float(d0 / idg::kSpeedOfLight);
         }
+        // host-streamed work groups: contiguous baseline ranges of <= kHostChunkBytes visibilities
+        {
+            const size_t bl_bytes = size_t(nr_timesteps) * nr_channels * 32;
+            size_t chunk = kHostChunkBytes;
+            if (const char *env = std::getenv("IDG_HOST_CHUNK_BYTES")) chunk = std::max<size_t>(1, std::strtoull(env, nullptr, 10));
+            const int32_t per = int32_t(std::max<size_t>(1, chunk / std::max<size_t>(1, bl_bytes)));
+            int64_t it = 0;
+            for (int32_t b0 = 0; b0 < nr_baselines; b0 += per) {
+                const int32_t b1 = std::min(nr_baselines, b0 + per);
+                const int64_t i0 = it;
+                while (it < int64_t(plan->items.size()) && plan->items[it].baseline < b1) ++it;
+                plan->groups.push_back(WorkGroup{b0, b1, i0, it});
+                plan->group_bytes = std::max(plan->group_bytes, size_t(b1 - b0) * bl_bytes);
+            }
+        }
         plan->order.resize(plan->items.size());
         std::iota(plan->order.begin(), plan->order.end(), 0);
         std::stable_sort(plan->order.begin(), plan->order.end(), [&](int32_t a, int32_t b) {
@@ -343,6 +402,14 @@ idg_status idg_workspace_size(const idg_plan *plan, size_t *bytes) {
     return IDG_OK;
 }
 
+idg_status idg_host_workspace_size(const idg_plan *plan, size_t *bytes) {
+    if (!plan || !bytes) return fail(IDG_ERR_INVALID_ARG, "NULL argument");
+    // kStagingBuffers staging buffers for gridding + as many for degridding (separate, so that the
+    // uploads of a grid call overlap a preceding degrid call and its downloads)
+    *bytes = size_t(2) * kStagingBuffers * plan->group_bytes;
+    return IDG_OK;
+}
+
 idg_status idg_grid(const idg_plan *plan, const void *d_vis, const float *d_uvw, const void *d_aterms,
                     const float *d_taper, void *d_grid, void *d_workspace, size_t workspace_bytes,
                     idg_stream stream) {
@@ -384,6 +451,119 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
         idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper, d_vis, const_cast<void *>(d_grid));
         cudaError_t e = idg::launch_degridder(a, s);
         if (e != cudaSuccess) return cuda_fail(e, "degridder launch");
+        return IDG_OK;
+    } catch (const std::exception &ex) {
+        return fail(IDG_ERR_INVALID_ARG, ex.what());
+    }
+}
+
+// ------------------------------------------------------------------------------------------------
+// Host-streamed calls: the paper's asynchronous I/O with triple buffering (Fig. 7).  Work
+// groups (contiguous baseline ranges) stream through kStagingBuffers device buffers; uploads run on a
+// copy stream, downloads on another, kernels on the caller's stream, ordered with events.
+// ------------------------------------------------------------------------------------------------
+idg_status idg_grid_host(const idg_plan *plan, const void *h_vis, const float *d_uvw, const void *d_aterms,
+                         const float *d_taper, void *d_grid, void *d_workspace, size_t workspace_bytes,
+                         idg_stream stream) {
+    try {
+        idg_status st = validate_call(plan, h_vis, d_uvw, d_aterms, d_taper, d_grid);
+        if (st != IDG_OK || plan->items.empty()) return st;
+        const size_t need = size_t(2) * kStagingBuffers * plan->group_bytes;
+        if (!d_workspace || workspace_bytes < need)
+            return fail(IDG_ERR_WORKSPACE_TOO_SMALL, "host-streamed gridding needs idg_host_workspace_size() = " +
+                                                         std::to_string(need) + " bytes");
+        const DeviceCopy *dc = nullptr;
+        if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        std::lock_guard<std::mutex> lock(*dc->pipeline_mu);
+        const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+        const size_t bl_bytes = size_t(plan->nr_timesteps) * plan->nr_channels * 32;
+        const int64_t bl_f2 = int64_t(plan->nr_timesteps) * plan->nr_channels * 4;  // float2 per baseline
+        char *staging = static_cast<char *>(d_workspace);                        // grid half of the workspace
+        cudaError_t e = cudaSuccess;
+        for (size_t gi = 0; gi < plan->groups.size() && e == cudaSuccess; ++gi) {
+            const WorkGroup &g = plan->groups[gi];
+            const int b = int(gi % kStagingBuffers);
+            char *buf = staging + size_t(b) * plan->group_bytes;
+            // the buffer is free once the gridder that last read it has finished
+            // (also across calls: an event never recorded is complete)
+            cudaStreamWaitEvent(dc->h2d, dc->ev_kernel_g[b], 0);
+            e = cudaMemcpyAsync(buf, static_cast<const char *>(h_vis) + size_t(g.b0) * bl_bytes,
+                                size_t(g.b1 - g.b0) * bl_bytes, cudaMemcpyHostToDevice, dc->h2d);
+            if (e != cudaSuccess) break;
+            cudaEventRecord(dc->ev_h2d[b], dc->h2d);
+            cudaStreamWaitEvent(s, dc->ev_h2d[b], 0);
+            if (g.i1 > g.i0) {
+                idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper,
+                                              reinterpret_cast<float2 *>(buf) - int64_t(g.b0) * bl_f2, d_grid);
+                a.order = dc->iota + g.i0;
+                a.nr_items = g.i1 - g.i0;
+                e = idg::launch_gridder(a, s);
+            }
+            cudaEventRecord(dc->ev_kernel_g[b], s);
+        }
+        if (e != cudaSuccess) return cuda_fail(e, "idg_grid_host");
+        return IDG_OK;
+    } catch (const std::exception &ex) {
+        return fail(IDG_ERR_INVALID_ARG, ex.what());
+    }
+}
+
+idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float *d_uvw, const void *d_aterms,
+                           const float *d_taper, void *h_vis, void *d_workspace, size_t workspace_bytes,
+                           idg_stream stream) {
+    try {
+        idg_status st = validate_call(plan, h_vis, d_uvw, d_aterms, d_taper, d_grid);
+        if (st != IDG_OK) return st;
+        const size_t need = size_t(2) * kStagingBuffers * plan->group_bytes;
+        if (!plan->groups.empty() && (!d_workspace || workspace_bytes < need))
+            return fail(IDG_ERR_WORKSPACE_TOO_SMALL, "host-streamed degridding needs idg_host_workspace_size() = " +
+                                                         std::to_string(need) + " bytes");
+        const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+        const size_t bl_bytes = size_t(plan->nr_timesteps) * plan->nr_channels * 32;
+        if (plan->items.empty()) {  // nothing to predict: every visibility is dropped -> 0
+            std::memset(h_vis, 0, size_t(plan->nr_baselines) * bl_bytes);
+            return IDG_OK;
+        }
+        const DeviceCopy *dc = nullptr;
+        if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        std::lock_guard<std::mutex> lock(*dc->pipeline_mu);
+        const int64_t bl_f2 = int64_t(plan->nr_timesteps) * plan->nr_channels * 4;
+        char *staging = static_cast<char *>(d_workspace) + size_t(kStagingBuffers) * plan->group_bytes;
+        cudaError_t e = cudaSuccess;
+        size_t last = 0;
+        for (size_t gi = 0; gi < plan->groups.size() && e == cudaSuccess; ++gi) {
+            const WorkGroup &g = plan->groups[gi];
+            const int b = int(gi % kStagingBuffers);
+            char *buf = staging + size_t(b) * plan->group_bytes;
+            const size_t bytes = size_t(g.b1 - g.b0) * bl_bytes;
+            // the buffer is free once its previous download has finished
+            cudaStreamWaitEvent(s, dc->ev_d2h[b], 0);
+            if (plan->nr_vis_dropped > 0) {
+                e = cudaMemsetAsync(buf, 0, bytes, s);  // dropped visibilities are 0 (R-12, R-13)
+                if (e != cudaSuccess) break;
+            }
+            if (g.i1 > g.i0) {
+                idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper,
+                                              reinterpret_cast<float2 *>(buf) - int64_t(g.b0) * bl_f2,
+                                              const_cast<void *>(d_grid));
+                a.order = dc->iota + g.i0;
+                a.nr_items = g.i1 - g.i0;
+                e = idg::launch_degridder(a, s);
+                if (e != cudaSuccess) break;
+            } else if (plan->nr_vis_dropped == 0) {
+                e = cudaMemsetAsync(buf, 0, bytes, s);
+                if (e != cudaSuccess) break;
+            }
+            cudaEventRecord(dc->ev_kernel_d[b], s);
+            cudaStreamWaitEvent(dc->d2h, dc->ev_kernel_d[b], 0);
+            e = cudaMemcpyAsync(static_cast<char *>(h_vis) + size_t(g.b0) * bl_bytes, buf, bytes,
+                                cudaMemcpyDeviceToHost, dc->d2h);
+            cudaEventRecord(dc->ev_d2h[b], dc->d2h);
+            last = gi;
+        }
+        if (e != cudaSuccess) return cuda_fail(e, "idg_degrid_host");
+        // completion of the call is observable on the caller's stream
+        for (int b = 0; b < kStagingBuffers && size_t(b) <= last; ++b) cudaStreamWaitEvent(s, dc->ev_d2h[b], 0);
         return IDG_OK;
     } catch (const std::exception &ex) {
         return fail(IDG_ERR_INVALID_ARG, ex.what());

@@ -45,7 +45,7 @@ _lib = None
 EXPORTED = ["idg_plan_create", "idg_plan_destroy", "idg_plan_nr_subgrids", "idg_plan_metadata",
             "idg_plan_stats", "idg_workspace_size", "idg_grid", "idg_degrid", "idg_rho_benchmark",
             "idg_profiling_enable", "idg_profiling_reset", "idg_profiling_read", "idg_launch_count",
-            "idg_kernel_variants",
+            "idg_kernel_variants", "idg_host_workspace_size", "idg_grid_host", "idg_degrid_host",
             "idg_status_string", "idg_last_error"]
 
 
@@ -68,6 +68,9 @@ def lib() -> ctypes.CDLL:
     L.idg_workspace_size.argtypes = [P, ctypes.POINTER(sz)]
     L.idg_grid.argtypes = [P, P, P, P, P, P, P, sz, P]
     L.idg_degrid.argtypes = [P, P, P, P, P, P, P, sz, P]
+    L.idg_host_workspace_size.argtypes = [P, ctypes.POINTER(sz)]
+    L.idg_grid_host.argtypes = [P, P, P, P, P, P, P, sz, P]
+    L.idg_degrid_host.argtypes = [P, P, P, P, P, P, P, sz, P]
     L.idg_rho_benchmark.argtypes = [i32, i32, P, ctypes.POINTER(ctypes.c_double),
                                     ctypes.POINTER(ctypes.c_double)]
     L.idg_profiling_enable.argtypes = [i32]
@@ -166,6 +169,11 @@ class Plan:
         _check(lib().idg_workspace_size(self._h, ctypes.byref(b)), "idg_workspace_size")
         return int(b.value)
 
+    def host_workspace_size(self) -> int:
+        b = ctypes.c_size_t()
+        _check(lib().idg_host_workspace_size(self._h, ctypes.byref(b)), "idg_host_workspace_size")
+        return int(b.value)
+
 
 # ------------------------------------------------------------------------------------------------
 # device calls (torch tensors are used only as device buffers)
@@ -217,6 +225,43 @@ def degrid(plan: Plan, grid_in, uvw, aterms, taper, vis_out, stream=None):
             _dev(vis_out, *sh["vis"], "vis")]
     _check(lib().idg_degrid(plan.handle, *args, None, 0, _stream(stream)), "idg_degrid")
     return vis_out
+
+
+def _host(t, dtype, shape, name):
+    import torch
+    if not isinstance(t, torch.Tensor) or t.is_cuda:
+        raise TypeError(f"{name} must be a CPU torch tensor (pinned for overlap)")
+    if t.dtype != dtype or tuple(t.shape) != tuple(shape) or not t.is_contiguous():
+        raise ValueError(f"{name} must be a contiguous {dtype} tensor of shape {tuple(shape)}")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def workspace(plan: Plan, device=None):
+    """A device workspace for the host-streamed calls (idg_host_workspace_size bytes)."""
+    import torch
+    return torch.empty(max(1, plan.host_workspace_size()), dtype=torch.uint8, device=device or "cuda")
+
+
+def grid_host(plan: Plan, vis_host, uvw, aterms, taper, grid_out, ws, stream=None):
+    """idg_grid_host: visibilities in (pinned) host memory, streamed through `ws`."""
+    sh = _shapes(plan)
+    args = [_host(vis_host, *sh["vis"], "vis_host"), _dev(uvw, *sh["uvw"], "uvw"),
+            _dev(aterms, *sh["aterms"], "aterms"), _dev(taper, *sh["taper"], "taper"),
+            _dev(grid_out, *sh["grid"], "grid")]
+    _check(lib().idg_grid_host(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)),
+           "idg_grid_host")
+    return grid_out
+
+
+def degrid_host(plan: Plan, grid_in, uvw, aterms, taper, vis_host_out, ws, stream=None):
+    """idg_degrid_host: predicted visibilities streamed back into (pinned) host memory."""
+    sh = _shapes(plan)
+    args = [_dev(grid_in, *sh["grid"], "grid"), _dev(uvw, *sh["uvw"], "uvw"),
+            _dev(aterms, *sh["aterms"], "aterms"), _dev(taper, *sh["taper"], "taper"),
+            _host(vis_host_out, *sh["vis"], "vis_host_out")]
+    _check(lib().idg_degrid_host(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(),
+                                 _stream(stream)), "idg_degrid_host")
+    return vis_host_out
 
 
 def rho_benchmark(rho: int = 17, iterations: int = 4096, stream=None) -> tuple[float, float]:

@@ -75,3 +75,14 @@ class ShardedIDG:
         from . import idg
         broadcast_grid(grid_in, src=src)
         return idg.degrid(self.plan, grid_in, uvw, aterms, taper, vis_out, stream=stream)
+
+    # host-streamed variants (visibilities in pinned host memory)
+    def grid_host(self, vis_host, uvw, aterms, taper, grid_out, ws, dst: int = 0, stream=None):
+        from . import idg
+        idg.grid_host(self.plan, vis_host, uvw, aterms, taper, grid_out, ws, stream=stream)
+        return reduce_grid(grid_out, dst=dst)
+
+    def degrid_host(self, grid_in, uvw, aterms, taper, vis_host_out, ws, src: int = 0, stream=None):
+        from . import idg
+        broadcast_grid(grid_in, src=src)
+        return idg.degrid_host(self.plan, grid_in, uvw, aterms, taper, vis_host_out, ws, stream=stream)
