@@ -191,3 +191,36 @@ def test_host_streamed_calls(name, kw, chunk, monkeypatch):
     idg.degrid_host(plan, G, uvw, at, tp, v_host, ws)
     torch.cuda.synchronize()
     assert torch.equal(v_host, v_dev.cpu())
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name,kw", [("ska", {}), ("predict", {})])
+def test_full_size_configs_sampled(name, kw):
+    """The SKA-low-shaped (N=8192, N~=32, C=32, T=8192: 2.9e9 visibilities, 94 GB) and predict-shaped
+    (512 stations, N=8192) configs at full size in the bench launch configuration: degridded
+    visibilities of sampled work items against the oracle, and the grid <-> degrid adjoint identity."""
+    obs = idgsynth.make_observation(name, **kw)
+    aterms = idgsynth.make_aterms(obs)
+    tap = idgsynth.make_taper(obs.subgrid_size)
+    plan = idg.Plan.from_observation(obs)
+    assert plan.stats()["nr_vis_dropped"] == 0
+    uvw, at, tp = _dev(obs.uvw), _dev(aterms), _dev(tap)
+    G = idgsynth.torch_grid(obs, "cuda")
+    V = idgsynth.torch_visibilities(obs, "cuda")
+    DG = torch.empty_like(V)
+    idg.degrid(plan, G, uvw, at, tp, DG)
+    gV = torch.zeros_like(G)
+    idg.grid(plan, V, uvw, at, tp, gV)
+    torch.cuda.synchronize()
+    lhs, rhs = _inner_t(DG, V), _inner_t(G, gV)
+    assert abs(lhs - rhs) / abs(lhs) < 1e-4, (lhs, rhs)
+    del V, gV
+    items = plan.metadata()
+    rng = np.random.default_rng(1)
+    sel = items[np.sort(rng.choice(len(items), 16, replace=False))]
+    sel = np.asarray(sel).astype(oracle.ITEM_DTYPE)
+    Gh = G.cpu().numpy()
+    ref = oracle.degrid(obs, sel, Gh, aterms, tap)
+    got = np.concatenate([DG[int(it["baseline"]), int(it["time_offset"]):int(it["time_offset"]) + int(it["nr_timesteps"]),
+                             int(it["channel_begin"]):int(it["channel_end"])].cpu().numpy().reshape(-1) for it in sel])
+    assert rel_rms(got, ref) <= TOL
