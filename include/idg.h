@@ -141,8 +141,11 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
  * events, so transfers overlap the kernels.  Semantics are those of idg_grid / idg_degrid:
  *   idg_grid_host    h_vis (read) -> d_grid (ACCUMULATED)
  *   idg_degrid_host  d_grid -> h_vis (OVERWRITTEN, dropped visibilities = 0)
- * d_workspace must hold idg_host_workspace_size() bytes (separate halves for the two directions, so a
- * grid call's uploads can overlap a preceding degrid call).  Both calls are asynchronous on `stream`;
+ * d_workspace must hold at least idg_host_workspace_size() bytes (three staging buffers per direction,
+ * in separate halves so a grid call's uploads can overlap a preceding degrid call).  A larger workspace
+ * gives more buffers per direction (workspace_bytes / (2 x work-group bytes), up to one per work group);
+ * with one per work group the uploads of a grid call never wait for kernels, so the next step's
+ * visibilities stream in while the current step degrids.  Both calls are asynchronous on `stream`;
  * h_vis must stay valid (and, for idg_grid_host, unmodified) until `stream` reaches the call's end.
  * Calls on the same plan are serialised internally (the pipeline streams and events belong to the
  * plan's device copy).

@@ -51,10 +51,9 @@ struct DeviceCopy {
     int32_t *iota = nullptr;       // plan order (work groups of the host-streamed calls)
     int32_t *baselines = nullptr;
     double *frequencies = nullptr;
-    // host-streamed pipeline: one copy stream per direction + per-buffer events
+    // host-streamed pipeline: one copy stream per direction + per-buffer events (grown on demand)
     cudaStream_t h2d = nullptr, d2h = nullptr;
-    cudaEvent_t ev_h2d[kStagingBuffers] = {}, ev_kernel_g[kStagingBuffers] = {};
-    cudaEvent_t ev_kernel_d[kStagingBuffers] = {}, ev_d2h[kStagingBuffers] = {};
+    std::vector<cudaEvent_t> *ev_h2d = nullptr, *ev_kernel_g = nullptr, *ev_kernel_d = nullptr, *ev_d2h = nullptr;
     std::mutex *pipeline_mu = nullptr;
 };
 
@@ -97,11 +96,10 @@ struct idg_plan {
             cudaFree(kv.second.iota);
             if (kv.second.h2d) cudaStreamDestroy(kv.second.h2d);
             if (kv.second.d2h) cudaStreamDestroy(kv.second.d2h);
-            for (int b = 0; b < kStagingBuffers; ++b) {
-                if (kv.second.ev_h2d[b]) cudaEventDestroy(kv.second.ev_h2d[b]);
-                if (kv.second.ev_kernel_g[b]) cudaEventDestroy(kv.second.ev_kernel_g[b]);
-                if (kv.second.ev_kernel_d[b]) cudaEventDestroy(kv.second.ev_kernel_d[b]);
-                if (kv.second.ev_d2h[b]) cudaEventDestroy(kv.second.ev_d2h[b]);
+            for (auto *v : {kv.second.ev_h2d, kv.second.ev_kernel_g, kv.second.ev_kernel_d, kv.second.ev_d2h}) {
+                if (!v) continue;
+                for (cudaEvent_t ev : *v) cudaEventDestroy(ev);
+                delete v;
             }
             delete kv.second.pipeline_mu;
             cudaFree(kv.second.baselines);
@@ -150,12 +148,10 @@ struct idg_plan {
         if ((e = cudaStreamCreateWithFlags(&dc.h2d, cudaStreamNonBlocking)) != cudaSuccess ||
             (e = cudaStreamCreateWithFlags(&dc.d2h, cudaStreamNonBlocking)) != cudaSuccess)
             return cuda_fail(e, "cudaStreamCreate(pipeline)");
-        for (int b = 0; b < kStagingBuffers; ++b) {
-            cudaEventCreateWithFlags(&dc.ev_h2d[b], cudaEventDisableTiming);
-            cudaEventCreateWithFlags(&dc.ev_kernel_g[b], cudaEventDisableTiming);
-            cudaEventCreateWithFlags(&dc.ev_kernel_d[b], cudaEventDisableTiming);
-            cudaEventCreateWithFlags(&dc.ev_d2h[b], cudaEventDisableTiming);
-        }
+        dc.ev_h2d = new std::vector<cudaEvent_t>();
+        dc.ev_kernel_g = new std::vector<cudaEvent_t>();
+        dc.ev_kernel_d = new std::vector<cudaEvent_t>();
+        dc.ev_d2h = new std::vector<cudaEvent_t>();
         dc.pipeline_mu = new std::mutex();
         if (!baselines.empty())
             cudaMemcpy(dc.baselines, baselines.data(), baselines.size() * 4, cudaMemcpyHostToDevice);
@@ -216,6 +212,23 @@ idg_status validate_call(const idg_plan *plan, const void *a, const void *b, con
     if (plan->items.empty()) return IDG_OK;
     if (!a || !b || !c || !d || !e) return fail(IDG_ERR_INVALID_ARG, "NULL device pointer");
     return IDG_OK;
+}
+
+// number of staging buffers per direction a workspace provides (>= kStagingBuffers), and events for them
+int staging_buffers(const idg_plan *plan, size_t workspace_bytes) {
+    if (plan->group_bytes == 0) return kStagingBuffers;
+    const size_t per_dir = workspace_bytes / (2 * plan->group_bytes);
+    return int(std::max<size_t>(kStagingBuffers, std::min<size_t>(per_dir, plan->groups.size())));
+}
+cudaError_t ensure_events(const DeviceCopy *dc, int n) {
+    for (auto *v : {dc->ev_h2d, dc->ev_kernel_g, dc->ev_kernel_d, dc->ev_d2h})
+        while (int(v->size()) < n) {
+            cudaEvent_t ev;
+            cudaError_t e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+            if (e != cudaSuccess) return e;
+            v->push_back(ev);
+        }
+    return cudaSuccess;
 }
 
 idg::KernelArgs make_args(const idg_plan *plan, const DeviceCopy *dc, const float *d_uvw,
@@ -478,20 +491,21 @@ idg_status idg_grid_host(const idg_plan *plan, const void *h_vis, const float *d
         const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
         const size_t bl_bytes = size_t(plan->nr_timesteps) * plan->nr_channels * 32;
         const int64_t bl_f2 = int64_t(plan->nr_timesteps) * plan->nr_channels * 4;  // float2 per baseline
+        const int nb = staging_buffers(plan, workspace_bytes);
         char *staging = static_cast<char *>(d_workspace);                        // grid half of the workspace
-        cudaError_t e = cudaSuccess;
+        cudaError_t e = ensure_events(dc, nb);
         for (size_t gi = 0; gi < plan->groups.size() && e == cudaSuccess; ++gi) {
             const WorkGroup &g = plan->groups[gi];
-            const int b = int(gi % kStagingBuffers);
+            const int b = int(gi % nb);
             char *buf = staging + size_t(b) * plan->group_bytes;
             // the buffer is free once the gridder that last read it has finished
             // (also across calls: an event never recorded is complete)
-            cudaStreamWaitEvent(dc->h2d, dc->ev_kernel_g[b], 0);
+            cudaStreamWaitEvent(dc->h2d, (*dc->ev_kernel_g)[b], 0);
             e = cudaMemcpyAsync(buf, static_cast<const char *>(h_vis) + size_t(g.b0) * bl_bytes,
                                 size_t(g.b1 - g.b0) * bl_bytes, cudaMemcpyHostToDevice, dc->h2d);
             if (e != cudaSuccess) break;
-            cudaEventRecord(dc->ev_h2d[b], dc->h2d);
-            cudaStreamWaitEvent(s, dc->ev_h2d[b], 0);
+            cudaEventRecord((*dc->ev_h2d)[b], dc->h2d);
+            cudaStreamWaitEvent(s, (*dc->ev_h2d)[b], 0);
             if (g.i1 > g.i0) {
                 idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper,
                                               reinterpret_cast<float2 *>(buf) - int64_t(g.b0) * bl_f2, d_grid);
@@ -499,7 +513,7 @@ idg_status idg_grid_host(const idg_plan *plan, const void *h_vis, const float *d
                 a.nr_items = g.i1 - g.i0;
                 e = idg::launch_gridder(a, s);
             }
-            cudaEventRecord(dc->ev_kernel_g[b], s);
+            cudaEventRecord((*dc->ev_kernel_g)[b], s);
         }
         if (e != cudaSuccess) return cuda_fail(e, "idg_grid_host");
         return IDG_OK;
@@ -528,16 +542,17 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
         if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
         std::lock_guard<std::mutex> lock(*dc->pipeline_mu);
         const int64_t bl_f2 = int64_t(plan->nr_timesteps) * plan->nr_channels * 4;
-        char *staging = static_cast<char *>(d_workspace) + size_t(kStagingBuffers) * plan->group_bytes;
-        cudaError_t e = cudaSuccess;
+        const int nb = staging_buffers(plan, workspace_bytes);
+        char *staging = static_cast<char *>(d_workspace) + size_t(nb) * plan->group_bytes;
+        cudaError_t e = ensure_events(dc, nb);
         size_t last = 0;
         for (size_t gi = 0; gi < plan->groups.size() && e == cudaSuccess; ++gi) {
             const WorkGroup &g = plan->groups[gi];
-            const int b = int(gi % kStagingBuffers);
+            const int b = int(gi % nb);
             char *buf = staging + size_t(b) * plan->group_bytes;
             const size_t bytes = size_t(g.b1 - g.b0) * bl_bytes;
             // the buffer is free once its previous download has finished
-            cudaStreamWaitEvent(s, dc->ev_d2h[b], 0);
+            cudaStreamWaitEvent(s, (*dc->ev_d2h)[b], 0);
             if (plan->nr_vis_dropped > 0) {
                 e = cudaMemsetAsync(buf, 0, bytes, s);  // dropped visibilities are 0 (R-12, R-13)
                 if (e != cudaSuccess) break;
@@ -554,16 +569,16 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
                 e = cudaMemsetAsync(buf, 0, bytes, s);
                 if (e != cudaSuccess) break;
             }
-            cudaEventRecord(dc->ev_kernel_d[b], s);
-            cudaStreamWaitEvent(dc->d2h, dc->ev_kernel_d[b], 0);
+            cudaEventRecord((*dc->ev_kernel_d)[b], s);
+            cudaStreamWaitEvent(dc->d2h, (*dc->ev_kernel_d)[b], 0);
             e = cudaMemcpyAsync(static_cast<char *>(h_vis) + size_t(g.b0) * bl_bytes, buf, bytes,
                                 cudaMemcpyDeviceToHost, dc->d2h);
-            cudaEventRecord(dc->ev_d2h[b], dc->d2h);
+            cudaEventRecord((*dc->ev_d2h)[b], dc->d2h);
             last = gi;
         }
         if (e != cudaSuccess) return cuda_fail(e, "idg_degrid_host");
         // completion of the call is observable on the caller's stream
-        for (int b = 0; b < kStagingBuffers && size_t(b) <= last; ++b) cudaStreamWaitEvent(s, dc->ev_d2h[b], 0);
+        for (int b = 0; b < nb && size_t(b) <= last; ++b) cudaStreamWaitEvent(s, (*dc->ev_d2h)[b], 0);
         return IDG_OK;
     } catch (const std::exception &ex) {
         return fail(IDG_ERR_INVALID_ARG, ex.what());

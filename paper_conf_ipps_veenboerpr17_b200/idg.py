@@ -236,10 +236,15 @@ def _host(t, dtype, shape, name):
     return ctypes.c_void_p(t.data_ptr())
 
 
-def workspace(plan: Plan, device=None):
-    """A device workspace for the host-streamed calls (idg_host_workspace_size bytes)."""
+def workspace(plan: Plan, device=None, full: bool = False):
+    """A device workspace for the host-streamed calls: the minimum (idg_host_workspace_size, three
+    staging buffers per direction) or, with full=True, one staging buffer per work group and direction
+    (2 x the visibility bytes) so consecutive grid/degrid calls overlap completely."""
     import torch
-    return torch.empty(max(1, plan.host_workspace_size()), dtype=torch.uint8, device=device or "cuda")
+    n = plan.host_workspace_size()
+    if full:
+        n = max(n, 2 * plan.nr_baselines * plan.nr_timesteps * plan.nr_channels * 32 + (64 << 20))
+    return torch.empty(max(1, n), dtype=torch.uint8, device=device or "cuda")
 
 
 def grid_host(plan: Plan, vis_host, uvw, aterms, taper, grid_out, ws, stream=None):
