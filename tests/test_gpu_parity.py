@@ -135,8 +135,13 @@ def test_grid_accumulates_and_degrid_zeroes_dropped(kind):
     assert np.all(got[covered == 0] == 0)                              # dropped -> exactly 0
 
 
-def _inner_t(a, b):
-    return torch.vdot(a.reshape(-1).to(torch.complex128), b.reshape(-1).to(torch.complex128)).item()
+def _inner_t(a, b, chunk=1 << 26):
+    """sum conj(a) b in complex128, in chunks (the full-size arrays are up to 94 GB)."""
+    a, b = a.reshape(-1), b.reshape(-1)
+    acc = 0j
+    for i in range(0, a.numel(), chunk):
+        acc += torch.vdot(a[i:i + chunk].to(torch.complex128), b[i:i + chunk].to(torch.complex128)).item()
+    return acc
 
 
 @pytest.mark.parametrize("name", ["lofar_dde", "lofar"])
