@@ -63,6 +63,7 @@ __device__ __forceinline__ f2p sub2(f2p a, f2p b) {
 }
 
 // (x, y) -> f16x2 hi = rn(x, y) and lo = rn(x - hi, y - hi): x = hi + lo to ~22 significant bits.
+// Used for the B operands (once per batch / item).
 __device__ __forceinline__ void split2(float x, float y, uint32_t &hi, uint32_t &lo) {
     const __half2 h = __floats2half2_rn(x, y);
     const float2 hf = __half22float2(h);
@@ -70,6 +71,17 @@ __device__ __forceinline__ void split2(float x, float y, uint32_t &hi, uint32_t 
     const __half2 l = __floats2half2_rn(d.x, d.y);
     hi = h2_bits(h);
     lo = h2_bits(l);
+}
+
+// Phasor split (|x|, |y| <= 1, per pair, on the critical path): hi = x with the low 13 mantissa bits
+// cleared (LOP3 on the ALU pipe; exactly representable in f16 for |x| >= 2^-14, and within 2^-25
+// otherwise), lo = x - hi (one FADD2, exact) -> f16.  |lo| < 2^-10 |x|, so x = hi + lo to ~21 bits.
+__device__ __forceinline__ void split_phasor(float x, float y, uint32_t &hi, uint32_t &lo) {
+    const float hx = __uint_as_float(__float_as_uint(x) & 0xffffe000u);
+    const float hy = __uint_as_float(__float_as_uint(y) & 0xffffe000u);
+    const float2 d = unpk(sub2(pk(x, y), pk(hx, hy)));
+    hi = h2_bits(__floats2half2_rn(hx, hy));
+    lo = h2_bits(__floats2half2_rn(d.x, d.y));
 }
 
 __device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
@@ -270,6 +282,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
                 const uint4 bf = frag_s[(kb - kb0) * 32 + lane];
                 const float4 df = dfk_s[(kb - kb0) * 4 + q];
                 const f2p dq = pk(df.x, df.y), dq4 = pk(df.z, df.w);
+                uint32_t ah[MT][4], al[MT][4];
 #pragma unroll
                 for (int i = 0; i < MT; ++i) {
                     const float2 ph0 = unpk(fma2(dq, Qv[i], Bv[i]));   // (row g, row g+8) at slot q
@@ -287,11 +300,16 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
                         __sincosf(ph1.x, &sn[2], &cs[2]);
                         __sincosf(ph1.y, &sn[3], &cs[3]);
                     }
-                    uint32_t ah[4], al[4];
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) split2(cs[j], sn[j], ah[j], al[j]);
-                    mma3(part[i], ah, al, bf);
+                    for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[i][j], al[i][j]);
                 }
+                // pass-major issue: consecutive mma are independent (different tiles)
+#pragma unroll
+                for (int i = 0; i < MT; ++i) mma16816(part[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
+#pragma unroll
+                for (int i = 0; i < MT; ++i) mma16816(part[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
+#pragma unroll
+                for (int i = 0; i < MT; ++i) mma16816(part[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
             }
         }
 #pragma unroll
@@ -425,6 +443,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
             const uint4 bf = frag_s[kb * 32 + lane];
             const float4 lm = lmn_s[(kb * 4 + q) * 2], nn = lmn_s[(kb * 4 + q) * 2 + 1];
             const f2p l2 = pk(lm.x, lm.y), m2 = pk(lm.z, lm.w), n2 = pk(nn.x, nn.y);
+            uint32_t ah[MT][4], al[MT][4];
 #pragma unroll
             for (int i = 0; i < MT; ++i) {
                 // phases of (row, slot q) and (row, slot q+4) in one FFMA2 chain per row
@@ -435,11 +454,15 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
                 __sincosf(p1.x, &sn[1], &cs[1]);  // row g+8, slot q
                 __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
                 __sincosf(p1.y, &sn[3], &cs[3]);  // row g+8, slot q+4
-                uint32_t ah[4], al[4];
 #pragma unroll
-                for (int j = 0; j < 4; ++j) split2(cs[j], sn[j], ah[j], al[j]);
-                mma3(acc[i], ah, al, bf);
+                for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[i][j], al[i][j]);
             }
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
         }
 #pragma unroll
         for (int i = 0; i < MT; ++i) {
