@@ -1,0 +1,90 @@
+// loop_probe.cu -- attribute the cost of the tensor-core gridder inner loop (design probe).
+// Per k-block per thread: MT tiles x {4 phases (FFMA2 x2), 4 sincos, 4 splits, 3 mma}.  Variants
+// drop parts to see which one binds.  Grid = 148 x BPS blocks of W warps, no memory traffic.
+#include <cstdio>
+#include <cstdint>
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+typedef unsigned long long u64;
+__device__ __forceinline__ u64 pk(float a, float b) { u64 r; asm("mov.b64 %0, {%1,%2};" : "=l"(r) : "f"(a), "f"(b)); return r; }
+__device__ __forceinline__ float2 up(u64 v) { float2 r; asm("mov.b64 {%0,%1}, %2;" : "=f"(r.x), "=f"(r.y) : "l"(v)); return r; }
+__device__ __forceinline__ u64 fma2(u64 a, u64 b, u64 c) { u64 r; asm("fma.rn.f32x2 %0,%1,%2,%3;" : "=l"(r) : "l"(a), "l"(b), "l"(c)); return r; }
+__device__ __forceinline__ u64 sub2(u64 a, u64 b) { u64 r; asm("sub.rn.f32x2 %0,%1,%2;" : "=l"(r) : "l"(a), "l"(b)); return r; }
+__device__ __forceinline__ uint32_t h2b(__half2 h) { return *reinterpret_cast<uint32_t *>(&h); }
+__device__ __forceinline__ void split(float x, float y, uint32_t &hi, uint32_t &lo) {
+    float hx = __uint_as_float(__float_as_uint(x) & 0xffffe000u), hy = __uint_as_float(__float_as_uint(y) & 0xffffe000u);
+    float2 d = up(sub2(pk(x, y), pk(hx, hy)));
+    hi = h2b(__floats2half2_rn(hx, hy)); lo = h2b(__floats2half2_rn(d.x, d.y));
+}
+__device__ __forceinline__ void mma(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+    asm("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3},{%4,%5,%6,%7},{%8,%9},{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3]) : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+// MODE bits: 1 = sincos, 2 = split, 4 = mma
+template <int MT, int MODE>
+__global__ void loop(float *out, int iters) {
+    const int lane = threadIdx.x & 31;
+    u64 B[MT], Q[MT];
+    float acc[MT][4];
+    for (int i = 0; i < MT; ++i) { B[i] = pk(0.1f * i + lane * 1e-3f, 0.2f); Q[i] = pk(0.3f, 0.4f + i * 1e-2f); for (int j = 0; j < 4; ++j) acc[i][j] = 0; }
+    uint32_t b0 = 0x3c003c00u ^ lane, b1 = 0x3c003c01u, b2 = 0x3c013c00u, b3 = lane;
+    u64 dq = pk(1e-3f, 2e-3f), dq4 = pk(3e-3f, 4e-3f);
+    for (int it = 0; it < iters; ++it) {
+        dq = fma2(dq, pk(1.0000001f, 1.0000001f), pk(1e-7f, 1e-7f));
+        uint32_t ah[MT][4], al[MT][4];
+#pragma unroll
+        for (int i = 0; i < MT; ++i) {
+            float2 p0 = up(fma2(dq, Q[i], B[i])), p1 = up(fma2(dq4, Q[i], B[i]));
+            float ph[4] = {p0.x, p0.y, p1.x, p1.y}, sn[4], cs[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                if (MODE & 1) __sincosf(ph[j], &sn[j], &cs[j]); else { sn[j] = ph[j] * 0.5f; cs[j] = ph[j] + 0.25f; }
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                if (MODE & 2) split(cs[j], sn[j], ah[i][j], al[i][j]);
+                else { ah[i][j] = __float_as_uint(cs[j]); al[i][j] = __float_as_uint(sn[j]); }
+            }
+        }
+        if (MODE & 4) {
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma(acc[i], ah[i], b0, b1);
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma(acc[i], ah[i], b2, b3);
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma(acc[i], al[i], b0, b1);
+        } else {
+#pragma unroll
+            for (int i = 0; i < MT; ++i)
+#pragma unroll
+                for (int j = 0; j < 4; ++j) acc[i][j] += __uint_as_float(ah[i][j] ^ al[i][j]);
+        }
+    }
+    float s = 0; for (int i = 0; i < MT; ++i) for (int j = 0; j < 4; ++j) s += acc[i][j];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+template <int MT, int MODE>
+void run(const char *name, int warps, int bps, float *out) {
+    const int iters = 2048;
+    const int blocks = 148 * bps, threads = 32 * warps;
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    loop<MT, MODE><<<blocks, threads>>>(out, 16); cudaDeviceSynchronize();
+    cudaEventRecord(e0); loop<MT, MODE><<<blocks, threads>>>(out, iters); cudaEventRecord(e1); cudaEventSynchronize(e1);
+    float ms; cudaEventElapsedTime(&ms, e0, e1);
+    double pairs = double(blocks) * threads * iters * MT * 4;
+    int clk; cudaDeviceGetAttribute(&clk, cudaDevAttrClockRate, 0);
+    printf("%-34s warps/SM %3d: %6.2f pairs/clk/SM\n", name, warps * bps, pairs / (ms * 1e-3) / 148 / 1.965e9);
+}
+int main() {
+    float *out; cudaMalloc(&out, 148 * 64 * 1024 * 4);
+    for (int bps : {1, 2, 3}) {
+        run<3, 7>("full (sincos+split+mma) MT3 W12", 12, bps, out);
+        run<3, 3>("sincos+split, no mma MT3 W12", 12, bps, out);
+        run<3, 5>("sincos+mma, no split MT3 W12", 12, bps, out);
+        run<3, 1>("sincos only MT3 W12", 12, bps, out);
+        run<3, 6>("split+mma, no sincos MT3 W12", 12, bps, out);
+    }
+    run<6, 7>("full MT6 W6", 6, 4, out);
+    run<2, 7>("full MT2 W8", 8, 4, out);
+    printf("%s\n", cudaGetErrorString(cudaGetLastError()));
+}
