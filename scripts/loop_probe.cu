@@ -31,6 +31,7 @@ __global__ void loop(float *out, int iters) {
     u64 dq = pk(1e-3f, 2e-3f), dq4 = pk(3e-3f, 4e-3f);
     for (int it = 0; it < iters; ++it) {
         dq = fma2(dq, pk(1.0000001f, 1.0000001f), pk(1e-7f, 1e-7f));
+        dq4 = fma2(dq4, pk(1.0000001f, 1.0000001f), pk(2e-7f, 2e-7f));
         uint32_t ah[MT][4], al[MT][4];
 #pragma unroll
         for (int i = 0; i < MT; ++i) {
