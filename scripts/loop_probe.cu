@@ -16,6 +16,17 @@ __device__ __forceinline__ void split(float x, float y, uint32_t &hi, uint32_t &
     float2 d = up(sub2(pk(x, y), pk(hx, hy)));
     hi = h2b(__floats2half2_rn(hx, hy)); lo = h2b(__floats2half2_rn(d.x, d.y));
 }
+// bf16 split without conversions: hi = upper halves (PRMT), lo = x - hi (FADD2), truncated by PRMT
+__device__ __forceinline__ void split_bf(float x, float y, uint32_t &hi, uint32_t &lo) {
+    hi = __byte_perm(__float_as_uint(x), __float_as_uint(y), 0x7632);
+    float hx = __uint_as_float(__float_as_uint(x) & 0xffff0000u), hy = __uint_as_float(__float_as_uint(y) & 0xffff0000u);
+    float2 d = up(sub2(pk(x, y), pk(hx, hy)));
+    lo = __byte_perm(__float_as_uint(d.x), __float_as_uint(d.y), 0x7632);
+}
+__device__ __forceinline__ void mma_bf(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+    asm("mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0,%1,%2,%3},{%4,%5,%6,%7},{%8,%9},{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3]) : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
 __device__ __forceinline__ void mma(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
     asm("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3},{%4,%5,%6,%7},{%8,%9},{%0,%1,%2,%3};"
         : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3]) : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
@@ -43,11 +54,19 @@ __global__ void loop(float *out, int iters) {
             }
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
-                if (MODE & 2) split(cs[j], sn[j], ah[i][j], al[i][j]);
+                if (MODE & 8) split_bf(cs[j], sn[j], ah[i][j], al[i][j]);
+                else if (MODE & 2) split(cs[j], sn[j], ah[i][j], al[i][j]);
                 else { ah[i][j] = __float_as_uint(cs[j]); al[i][j] = __float_as_uint(sn[j]); }
             }
         }
-        if (MODE & 4) {
+        if ((MODE & 4) && (MODE & 8)) {
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma_bf(acc[i], ah[i], b0, b1);
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma_bf(acc[i], ah[i], b2, b3);
+#pragma unroll
+            for (int i = 0; i < MT; ++i) mma_bf(acc[i], al[i], b0, b1);
+        } else if (MODE & 4) {
 #pragma unroll
             for (int i = 0; i < MT; ++i) mma(acc[i], ah[i], b0, b1);
 #pragma unroll
@@ -78,14 +97,16 @@ void run(const char *name, int warps, int bps, float *out) {
 }
 int main() {
     float *out; cudaMalloc(&out, 148 * 64 * 1024 * 4);
-    for (int bps : {1, 2, 3}) {
-        run<3, 7>("full (sincos+split+mma) MT3 W12", 12, bps, out);
-        run<3, 3>("sincos+split, no mma MT3 W12", 12, bps, out);
-        run<3, 5>("sincos+mma, no split MT3 W12", 12, bps, out);
-        run<3, 1>("sincos only MT3 W12", 12, bps, out);
-        run<3, 6>("split+mma, no sincos MT3 W12", 12, bps, out);
+    for (int bps : {2, 3}) {
+        run<3, 7>("f16 full (sincos+split+mma)", 12, bps, out);
+        run<3, 15>("bf16 full (sincos+PRMT split+mma)", 12, bps, out);
+        run<3, 14>("bf16 split+mma, no sincos", 12, bps, out);
+        run<3, 6>("f16 split+mma, no sincos", 12, bps, out);
+        run<3, 10>("bf16 split, no sincos/mma", 12, bps, out);
+        run<3, 2>("f16 split, no sincos/mma", 12, bps, out);
+        run<3, 1>("sincos only", 12, bps, out);
     }
-    run<6, 7>("full MT6 W6", 6, 4, out);
-    run<2, 7>("full MT2 W8", 8, 4, out);
+    run<2, 15>("bf16 full MT2 W8", 8, 4, out);
+    run<4, 15>("bf16 full MT4 W9", 9, 3, out);
     printf("%s\n", cudaGetErrorString(cudaGetLastError()));
 }
