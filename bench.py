@@ -90,6 +90,13 @@ class ClockSampler:
         if self._h is not None:
             self._t.join()
 
+    def energy_mj(self):
+        """Board energy counter (mJ since driver load; NVML), None if unavailable."""
+        try:
+            return self._nvml.nvmlDeviceGetTotalEnergyConsumption(self._h)
+        except Exception:
+            return None
+
     def summary(self):
         return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
                 "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
@@ -246,11 +253,13 @@ def run_ours(args):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clocks:
         barrier()
+        mj0 = clocks.energy_mj()
         ev0.record(stream)
         for _ in range(args.steps):
             step(vis_d, out_d)
         ev1.record(stream)
         barrier()
+        mj1 = clocks.energy_mj()
     idg.profiling_enable(False)
     gpu_launches = idg.launch_count() - launches0
     kern = idg.profiling_read()
@@ -264,6 +273,14 @@ def run_ours(args):
         dist.all_reduce(nvis_t)
     nvis_total = float(nvis_t.item())
     value = nvis_total * args.steps / (ms_max * 1e-3) / 1e6
+    # energy efficiency (Fig. 15: GFlops/W per kernel; here the whole step, board energy)
+    energy = None
+    if mj0 is not None and mj1 is not None and mj1 > mj0:
+        joules = (mj1 - mj0) / 1e3
+        ops = 2 * OPS_PER_PAIR * float(pairs) * args.steps       # grid + degrid pairs on this rank
+        energy = {"J_per_step": joules / args.steps, "avg_W": joules / (ms * 1e-3),
+                  "GOps_per_J": ops / joules / 1e9, "source": "NVML total energy counter, this GPU, timed region",
+                  "paper_context": "GTX 1080: 32 / 23 GFlops/W gridder / degridder (P:306)"}
 
     # ---- e2e: host buffers through the public API ------------------------------------------------
     # Every step uploads its inputs (visibilities, uvw) from pinned host memory and downloads the
@@ -388,7 +405,7 @@ def run_ours(args):
                    "l2": "inputs larger than L2 (visibilities 4 GB/step)"},
         "grid_mvis_s": (nvis_rank / (per_kernel["gridder"]["avg_ms"] * 1e-3) / 1e6) if "gridder" in per_kernel else None,
         "degrid_mvis_s": (nvis_rank / (per_kernel["degridder"]["avg_ms"] * 1e-3) / 1e6) if "degridder" in per_kernel else None,
-        "plan_s": plan_s, "clocks": clocks.summary(), "e2e": e2e, "gpu_launches": gpu_launches,
+        "plan_s": plan_s, "clocks": clocks.summary(), "energy": energy, "e2e": e2e, "gpu_launches": gpu_launches,
         "roofline": roofline, "kernels": per_kernel, "rho_sweep_TOps_s": rho_sweep or None,
         "cpu_baseline": cpu,
     }
