@@ -40,6 +40,8 @@ class Observation:
     w_offset: float              # w0 (wavelengths)
     seed: int
     aterm_kind: str = "identity"     # "identity" | "random"
+    nr_w_planes: int = 1             # W-stacking planes; 1 = none
+    w_step: float = 0.0              # plane spacing (wavelengths)
 
     @property
     def nr_baselines(self) -> int:
@@ -66,7 +68,7 @@ class Observation:
                     image_size=self.image_size, kernel_size=self.kernel_size,
                     max_timesteps_per_subgrid=self.max_timesteps_per_subgrid,
                     max_channels_per_subgrid=self.max_channels_per_subgrid,
-                    w_offset=self.w_offset)
+                    w_offset=self.w_offset, nr_w_planes=self.nr_w_planes, w_step=self.w_step)
 
     def subset(self, nr_baselines: int | None = None, nr_timesteps: int | None = None,
                baseline_begin: int = 0) -> "Observation":
@@ -180,7 +182,7 @@ def make_observation(name: str, **overrides) -> Observation:
     aterms, dt, w_offset, seed, ...) -- same recipe, same seed unless overridden."""
     cfg = dict(CONFIGS[name])
     for k, v in overrides.items():
-        if k not in cfg and k not in ("w_offset", "C_block"):
+        if k not in cfg and k not in ("w_offset", "C_block", "w_planes"):
             raise KeyError(k)
         cfg[k] = v
     rng = np.random.default_rng(cfg["seed"])
@@ -208,10 +210,15 @@ def make_observation(name: str, **overrides) -> Observation:
     w0 = cfg.get("w_offset", 0.0)
     if w0 == "half_median":
         w0 = 0.5 * float(np.median(np.abs(uvw[:, :, 2]))) * float(freqs[0]) / SPEED_OF_LIGHT
+    nz, w_step = int(cfg.get("w_planes", 1)), 0.0
+    if nz > 1:   # planes spanning the |w| range of the observation at the middle frequency
+        wmax = float(np.max(np.abs(uvw[:, :, 2]))) * float(freqs[len(freqs) // 2]) / SPEED_OF_LIGHT
+        w_step = 2.0 * wmax / nz
     return Observation(name=name, nr_stations=S, baselines=bl, uvw=uvw, frequencies=freqs,
                        aterm_offsets=offs, subgrid_size=cfg["Ns"], grid_size=cfg["N"], image_size=L,
                        kernel_size=cfg["K"], max_timesteps_per_subgrid=cfg["Tmax"],
-                       max_channels_per_subgrid=int(cfg.get("C_block", 0)), w_offset=float(w0), seed=cfg["seed"], aterm_kind=cfg["aterms"])
+                       max_channels_per_subgrid=int(cfg.get("C_block", 0)), w_offset=float(w0),
+                       nr_w_planes=nz, w_step=w_step, seed=cfg["seed"], aterm_kind=cfg["aterms"])
 
 
 # ----------------------------------------------------------------------------------------------
@@ -276,10 +283,11 @@ def make_visibilities(obs: Observation, seed_offset: int = 11) -> np.ndarray:
 
 
 def make_grid(obs: Observation, seed_offset: int = 13) -> np.ndarray:
-    """complex64 [4][N][N] random model grid (input of degridding)."""
+    """complex64 [4][N][N] (or [nz][4][N][N] with W-stacking) random model grid (degridding input)."""
     rng = np.random.default_rng(obs.seed + seed_offset)
     N = obs.grid_size
-    g = np.empty((4, N, N), dtype=np.complex64)
+    shape = (4, N, N) if obs.nr_w_planes <= 1 else (obs.nr_w_planes, 4, N, N)
+    g = np.empty(shape, dtype=np.complex64)
     f = g.view(np.float32)
     f[...] = rng.standard_normal(f.shape, dtype=np.float32) * np.float32(math.sqrt(0.5))
     return g

@@ -33,7 +33,8 @@ class _Params(ctypes.Structure):
     _fields_ = [("subgrid_size", ctypes.c_int32), ("grid_size", ctypes.c_int32),
                 ("image_size", ctypes.c_double), ("kernel_size", ctypes.c_int32),
                 ("max_timesteps_per_subgrid", ctypes.c_int32),
-                ("max_channels_per_subgrid", ctypes.c_int32), ("w_offset", ctypes.c_double)]
+                ("max_channels_per_subgrid", ctypes.c_int32), ("w_offset", ctypes.c_double),
+                ("nr_w_planes", ctypes.c_int32), ("w_step", ctypes.c_double)]
 
 
 def build(force: bool = False) -> str:
@@ -79,7 +80,8 @@ def _ptr(a: np.ndarray):
 def _params(p: dict) -> _Params:
     return _Params(int(p["subgrid_size"]), int(p["grid_size"]), float(p["image_size"]),
                    int(p["kernel_size"]), int(p["max_timesteps_per_subgrid"]),
-                   int(p["max_channels_per_subgrid"]), float(p["w_offset"]))
+                   int(p["max_channels_per_subgrid"]), float(p["w_offset"]),
+                   int(p.get("nr_w_planes", 1)), float(p.get("w_step", 0.0)))
 
 
 def _c(a, dtype):
@@ -140,11 +142,17 @@ def degridder_item(obs, item, subgrid, aterms, taper) -> np.ndarray:
     return out
 
 
-def grid(obs, items, vis, aterms, taper, grid_out: np.ndarray | None = None, nthreads: int = 0):
-    """Accumulate the gridded visibilities of `items` into a complex128 [4][N][N] grid."""
-    p = _params(obs.plan_params())
+def grid_shape(obs):
+    """[4][N][N], or [nz][4][N][N] with W-stacking (R-21)."""
+    nz = int(obs.plan_params().get("nr_w_planes", 1))
     N = obs.grid_size
-    g = np.zeros((4, N, N), dtype=np.complex128) if grid_out is None else grid_out
+    return (4, N, N) if nz <= 1 else (nz, 4, N, N)
+
+
+def grid(obs, items, vis, aterms, taper, grid_out: np.ndarray | None = None, nthreads: int = 0):
+    """Accumulate the gridded visibilities of `items` into a complex128 grid_shape(obs) grid."""
+    p = _params(obs.plan_params())
+    g = np.zeros(grid_shape(obs), dtype=np.complex128) if grid_out is None else grid_out
     assert g.dtype == np.complex128 and g.flags.c_contiguous
     it = _c(items, ITEM_DTYPE)
     uvw, fr, bl = _c(obs.uvw, np.float32), _c(obs.frequencies, np.float64), _c(obs.baselines, np.int32)

@@ -45,11 +45,26 @@ def check_plan(obs, items, nr_dropped, check_maximal=True):
         cu = (uu.max() + uu.min()) / 2 + N / 2
         cv = (vv.max() + vv.min()) / 2 + N / 2
         assert abs(x + n / 2 - cu) <= 0.5 + 1e-9 and abs(y + n / 2 - cv) <= 0.5 + 1e-9
+        nz = getattr(obs, "nr_w_planes", 1)
+        if nz > 1:   # R-21: every timestep's w lies in the item's plane interval (edge planes unbounded)
+            z = int(it["z"])
+            assert 0 <= z < nz
+            nu_ref = obs.frequencies[c0 + (c1 - c0) // 2]
+            w = obs.uvw[b, t0:t0 + nt, 2].astype(np.float64) * nu_ref / C0
+            w0 = obs.w_offset + (z - (nz - 1) / 2) * obs.w_step
+            lo = -np.inf if z == 0 else w0 - obs.w_step / 2 - 1e-9 * obs.w_step
+            hi = np.inf if z == nz - 1 else w0 + obs.w_step / 2 + 1e-9 * obs.w_step
+            assert np.all((w >= lo) & (w <= hi)), (it, w.min(), w.max(), lo, hi)
+        else:
+            assert int(it["z"]) == 0
         if check_maximal:
             te = t0 + nt
             if te < T and te < offs[slot + 1] and nt < obs.max_timesteps_per_subgrid:
                 uu, vv = u[b, t0:te + 1, c0:c1], v[b, t0:te + 1, c0:c1]
                 fits = (uu.max() - uu.min()) + K <= n and (vv.max() - vv.min()) + K <= n
+                if nz > 1:   # the next timestep may also start a new W-plane
+                    wn = float(obs.uvw[b, te, 2]) * nu_ref / C0
+                    fits = fits and (lo <= wn <= hi)
                 assert not fits, f"item {it} is not maximal"
     assert cover.max(initial=0) <= 1, "visibility in two items"
     assert int((cover == 0).sum()) == nr_dropped, (int((cover == 0).sum()), nr_dropped)

@@ -208,3 +208,46 @@ def test_off_cell_visibility_spreads_as_dirichlet_kernel():
     want = dirichlet(v_rel - k)[:, None] * dirichlet(u_rel - k)[None, :]
     for pol in range(4):
         np.testing.assert_allclose(sub[pol], complex(vis[0, 0, 0, pol]) * want, rtol=1e-10, atol=1e-10)
+
+
+# ------------------------------------------------------------------------------------------------
+# W-stacking (reading R-21): per-plane w0 and grid copies
+# ------------------------------------------------------------------------------------------------
+
+def test_w_stacking_point_source_matches_eq1_with_full_w_term():
+    """With W-planes the model of plane z carries exp(-2 pi i w0_z n0); degridding every item from its
+    own plane then reproduces Eq. (1) with the FULL w-term (no w0 left)."""
+    obs = idgsynth.make_observation("small_dde", w_planes=4)
+    assert obs.nr_w_planes == 4
+    items, dropped = oracle.plan(obs)
+    assert dropped == 0 and len(set(items["z"].tolist())) >= 3
+    items = items[::5]
+    taper = idgsynth.make_taper(obs.subgrid_size)
+    aterms = idgsynth.make_aterms(obs, "random")
+    B = np.array([[0.7 + 0.1j, -0.3j], [0.2, 1.1 - 0.4j]])
+    x0, y0 = 10, 5
+    g1, (l0, m0, n0) = _point_source_case(obs, x0, y0, B, taper, aterms)
+    nz = obs.nr_w_planes
+    w0s = obs.w_offset + (np.arange(nz) - (nz - 1) / 2) * obs.w_step
+    grid = np.stack([g1 * np.exp(-2j * np.pi * w0 * n0) for w0 in w0s])
+    got = oracle.degrid(obs, items, grid, aterms, taper)
+    flat = dataclasses.replace(obs, w_offset=0.0)           # Eq. (1) with the full w-term
+    want = _eq1_visibilities(flat, items, aterms, x0, y0, B, (l0, m0, n0))
+    err = np.linalg.norm(got - want) / np.linalg.norm(want)
+    assert err < 1e-11, err
+
+
+def test_w_stacking_adjoint_identity():
+    obs = idgsynth.make_observation("small_dde", w_planes=3)
+    items, _ = oracle.plan(obs)
+    items = items[::3]
+    taper = idgsynth.make_taper(obs.subgrid_size)
+    aterms = idgsynth.make_aterms(obs, "random")
+    vis = idgsynth.make_visibilities(obs)
+    G = idgsynth.make_grid(obs)
+    assert G.shape[0] == 3
+    DG = oracle.degrid(obs, items, G, aterms, taper)
+    V = oracle.gather_visibilities(obs, items, vis).astype(np.complex128)
+    gV = oracle.grid(obs, items, vis, aterms, taper)
+    lhs, rhs = _inner(DG, V), _inner(G.astype(np.complex128), gV)
+    assert abs(lhs - rhs) / abs(lhs) < 1e-12, (lhs, rhs)

@@ -48,3 +48,11 @@ def test_plan_respects_tmax_and_slots():
     assert items["nr_timesteps"].max() == obs.max_timesteps_per_subgrid
     # slot boundaries every 256 steps: items split there even when they would fit
     assert set(items["time_offset"].tolist()) >= {0, 256, 512}
+
+
+@pytest.mark.parametrize("nz", [2, 5])
+def test_plan_w_planes(nz):
+    obs = idgsynth.make_observation("small_dde", w_planes=nz)
+    items, dropped = oracle.plan(obs)
+    check_plan(obs, items, dropped)
+    assert len(set(items["z"].tolist())) >= 2
