@@ -54,6 +54,11 @@ typedef struct {
     int32_t max_timesteps_per_subgrid; /* T~max >= 1 (R-14)                                   */
     int32_t max_channels_per_subgrid;  /* C~: channel block size; 0 = all channels (R-9)     */
     double w_offset;                   /* w0 (wavelengths) subtracted in the w-term           */
+    int32_t nr_w_planes;               /* W-stacking: number of W-planes; 0 or 1 = none */
+    double w_step;                     /* W-plane spacing (wavelengths), > 0 when nr_w_planes > 1.   */
+                                       /* Plane z has w0_z = w_offset + (z - (nz-1)/2) w_step; each  */
+                                       /* item lies in the plane nearest to w at its block's middle  */
+                                       /* channel (clamped) and never straddles a plane (R-21).       */
 } idg_plan_params;
 
 /* One work item = one subgrid and its visibilities.  Bit-exact with the oracle's plan. */
@@ -65,7 +70,7 @@ typedef struct {
     int32_t channel_end;               /* c1 (exclusive)                                            */
     int32_t aterm_index;               /* A-term slot of t0 (R-15)                                  */
     int32_t x, y;                      /* subgrid corner in grid cells; centre cell x+N~/2 (R-11)   */
-    int32_t z;                         /* W-plane index; always 0 (no W-stacking yet)              */
+    int32_t z;                         /* W-plane index (0 without W-stacking, R-21)               */
 } idg_metadata;
 
 typedef struct idg_plan idg_plan;
@@ -113,7 +118,8 @@ idg_status idg_workspace_size(const idg_plan *plan, size_t *bytes);
  *   d_uvw      float32 [nbl][T][3] metres (the same values the plan was built from)
  *   d_aterms   complex64 [slots][S][N~][N~][4] (Jones matrices per station and subgrid pixel)
  *   d_taper    float32 [N~][N~] (spheroidal)
- *   d_grid     complex64 [4][N][N], ACCUMULATED (+=); subgrid sums use fp32 atomics, so the order of
+ *   d_grid     complex64 [nz][4][N][N] (nz = W-planes, 1 without W-stacking), ACCUMULATED (+=);
+ *              subgrid sums use fp32 atomics, so the order of
  *              additions (not the math) is unspecified (R-19)
  *   d_workspace, workspace_bytes   >= idg_workspace_size (may be NULL/0 when that is 0)
  * Only the visibilities in the plan's items are read.
@@ -125,7 +131,7 @@ idg_status idg_grid(const idg_plan *plan, const void *d_vis, const float *d_uvw,
 /*
  * idg_degrid -- degridding: splitter -> subgrid inverse FFT -> taper/A-term (Alg. 2
  * lines 2-3) -> degridder (Alg. 2), fused into one sm_100a kernel per work item.
- *   d_grid     complex64 [4][N][N] model grid (read only)
+ *   d_grid     complex64 [nz][4][N][N] model grid (read only)
  *   d_vis      complex64 [nbl][T][C][4], OVERWRITTEN; dropped visibilities are set to 0
  *   other arguments as idg_grid.
  */

@@ -203,6 +203,10 @@ idg_status validate_params(const idg_plan_params *p) {
     if (p->max_channels_per_subgrid < 0)
         return fail(IDG_ERR_INVALID_ARG, "max_channels_per_subgrid must be >= 0");
     if (!std::isfinite(p->w_offset)) return fail(IDG_ERR_INVALID_ARG, "w_offset is not finite");
+    if (p->nr_w_planes < 0 || p->nr_w_planes > 4096)
+        return fail(IDG_ERR_INVALID_ARG, "nr_w_planes must be in [0, 4096]");
+    if (p->nr_w_planes > 1 && !(p->w_step > 0.0 && std::isfinite(p->w_step)))
+        return fail(IDG_ERR_INVALID_ARG, "w_step must be positive and finite when nr_w_planes > 1");
     return IDG_OK;
 }
 
@@ -240,6 +244,8 @@ idg::KernelArgs make_args(const idg_plan *plan, const DeviceCopy *dc, const floa
     a.cell_l = float(p.image_size / p.subgrid_size);
     a.inv_image_size = 1.0 / p.image_size;
     a.w_offset = p.w_offset;
+    a.nr_w_planes = p.nr_w_planes > 1 ? p.nr_w_planes : 1;
+    a.w_step = p.nr_w_planes > 1 ? p.w_step : 0.0;
     a.nr_stations = plan->nr_stations;
     a.nr_baselines = plan->nr_baselines;
     a.nr_timesteps = plan->nr_timesteps;

@@ -82,7 +82,7 @@ __device__ __forceinline__ ItemSetup item_setup(const KernelArgs &a, int item, i
     s.st2 = a.baselines[2 * s.md.baseline + 1];
     s.u0 = double(s.md.x + NS / 2 - a.grid_size / 2) * a.inv_image_size;
     s.v0 = double(s.md.y + NS / 2 - a.grid_size / 2) * a.inv_image_size;
-    s.w0 = a.w_offset;
+    s.w0 = a.w_offset + (double(s.md.z) - double(a.nr_w_planes - 1) / 2.0) * a.w_step;  // W-plane (R-21)
     s.f_ref = a.frequencies[s.md.channel_begin + s.nc / 2] / kSpeedOfLight;
     return s;
 }
@@ -172,7 +172,7 @@ __device__ __forceinline__ void gridder_epilogue(const KernelArgs &a, const Item
             idx += step;
             idx -= (idx >= NS) ? NS : 0;
         }
-        float2 *dst = a.grid + (int64_t(pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx;
+        float2 *dst = a.grid + ((int64_t(md.z) * 4 + pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx;
         red_add(dst, sum);
     }
 }
@@ -188,7 +188,7 @@ __device__ __forceinline__ void degridder_split_columns(const KernelArgs &a, con
     const idg_metadata &md = s.md;
     for (int o = threadIdx.x; o < 4 * NPIX; o += nt) {
         const int pol = o / NPIX, rem = o - pol * NPIX, ky = rem / NS, kx = rem - ky * NS;
-        sub_s[o] = a.grid[(int64_t(pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx];
+        sub_s[o] = a.grid[((int64_t(md.z) * 4 + pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx];
     }
     init_twiddles<NS>(tw, +1.0f);
     __syncthreads();

@@ -32,7 +32,9 @@ struct KernelArgs {
     int32_t grid_size;           // N
     float cell_l;                // L / N~   (direction-cosine step of a subgrid pixel)
     double inv_image_size;       // du = 1/L (wavelengths per grid cell)
-    double w_offset;             // w0
+    double w_offset;             // w0 (centre of the W-planes)
+    int32_t nr_w_planes;         // >= 1
+    double w_step;               // W-plane spacing (wavelengths)
     int32_t nr_stations, nr_baselines, nr_timesteps, nr_channels;
     int64_t nr_items;
     const idg_metadata *items;   // [nr_items]

@@ -33,7 +33,8 @@ class PlanParams(ctypes.Structure):
     _fields_ = [("subgrid_size", ctypes.c_int32), ("grid_size", ctypes.c_int32),
                 ("image_size", ctypes.c_double), ("kernel_size", ctypes.c_int32),
                 ("max_timesteps_per_subgrid", ctypes.c_int32),
-                ("max_channels_per_subgrid", ctypes.c_int32), ("w_offset", ctypes.c_double)]
+                ("max_channels_per_subgrid", ctypes.c_int32), ("w_offset", ctypes.c_double),
+                ("nr_w_planes", ctypes.c_int32), ("w_step", ctypes.c_double)]
 
 
 class KernelTime(ctypes.Structure):
@@ -109,10 +110,12 @@ class Plan:
 
     def __init__(self, *, subgrid_size: int, grid_size: int, image_size: float, kernel_size: int,
                  max_timesteps_per_subgrid: int, max_channels_per_subgrid: int = 0, w_offset: float = 0.0,
+                 nr_w_planes: int = 1, w_step: float = 0.0,
                  nr_stations: int, uvw: np.ndarray, frequencies: np.ndarray, baselines: np.ndarray,
                  aterm_offsets: np.ndarray):
         self.params = PlanParams(subgrid_size, grid_size, image_size, kernel_size, max_timesteps_per_subgrid,
-                                 max_channels_per_subgrid, w_offset)
+                                 max_channels_per_subgrid, w_offset, nr_w_planes, w_step)
+        self.nr_w_planes = max(1, int(nr_w_planes))
         uvw = _np(uvw, np.float32)
         freqs = _np(frequencies, np.float64)
         bl = _np(baselines, np.int32)
@@ -205,7 +208,8 @@ def _shapes(plan: Plan):
                 uvw=(torch.float32, (plan.nr_baselines, plan.nr_timesteps, 3)),
                 aterms=(torch.complex64, (plan.nr_aterm_slots, plan.nr_stations, n, n, 4)),
                 taper=(torch.float32, (n, n)),
-                grid=(torch.complex64, (4, plan.grid_size, plan.grid_size)))
+                grid=(torch.complex64, (4, plan.grid_size, plan.grid_size) if plan.nr_w_planes == 1
+                      else (plan.nr_w_planes, 4, plan.grid_size, plan.grid_size)))
 
 
 def grid(plan: Plan, vis, uvw, aterms, taper, grid_out, stream=None):

@@ -58,7 +58,9 @@ def _plans_equal(obs):
 @pytest.mark.parametrize("name,kw", [("tiny", {}), ("small_dde", {}), ("small_dde", dict(C=7, C_block=3)),
                                      ("lofar", dict(T=2048, nr_stations=16)),
                                      ("ska", dict(T=768, nr_stations=12)),
-                                     ("predict", dict(T=256, nr_stations=14))])
+                                     ("predict", dict(T=256, nr_stations=14)),
+                                     ("small_dde", dict(w_planes=4)),
+                                     ("lofar_dde", dict(T=1024, nr_stations=12, w_planes=8))])
 def test_plan_bit_exact_with_oracle(name, kw):
     obs = idgsynth.make_observation(name, **kw)
     items, st = _plans_equal(obs)
@@ -87,7 +89,8 @@ def test_plan_argument_validation():
               baselines=obs.baselines, aterm_offsets=obs.aterm_offsets)
     bad = [dict(subgrid_size=20), dict(grid_size=16), dict(image_size=-1.0), dict(kernel_size=16),
            dict(max_timesteps_per_subgrid=0), dict(aterm_offsets=np.array([0, 10], dtype=np.int32)),
-           dict(frequencies=-obs.frequencies), dict(baselines=obs.baselines[:, ::-1].copy())]
+           dict(frequencies=-obs.frequencies), dict(baselines=obs.baselines[:, ::-1].copy()),
+           dict(nr_w_planes=4, w_step=0.0), dict(nr_w_planes=-1)]
     for b in bad:
         with pytest.raises(idg.IDGError) as e:
             idg.Plan(**{**kw, **b})

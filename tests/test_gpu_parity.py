@@ -38,8 +38,7 @@ def _dev(a):
 
 def gpu_grid(obs, vis, aterms, taper, plan=None):
     plan = plan or idg.Plan.from_observation(obs)
-    N = obs.grid_size
-    g = torch.zeros((4, N, N), dtype=torch.complex64, device="cuda")
+    g = torch.zeros(oracle.grid_shape(obs), dtype=torch.complex64, device="cuda")
     idg.grid(plan, _dev(vis), _dev(obs.uvw), _dev(aterms), _dev(taper), g)
     torch.cuda.synchronize()
     return g
@@ -66,6 +65,8 @@ CASES = [
     ("ska", dict(T=384, nr_stations=4), None, "spheroidal"),         # N~=32, N=8192, 32 ch
     ("predict", dict(T=256, nr_stations=4, C=8), None, "spheroidal"),  # N~=32, 8 ch: one k-block/timestep
     ("small_dde", dict(C=24, C_block=8), None, "spheroidal"),       # 3 channel blocks of 8
+    ("small_dde", dict(w_planes=4), None, "spheroidal"),            # W-stacking (NEXT-1, R-21)
+    ("lofar_dde", dict(T=512, nr_stations=5, w_planes=3), None, "spheroidal"),
 ]
 
 
@@ -173,7 +174,8 @@ def test_full_size_adjoint_and_sampled_items(name, kind):
 
 
 @pytest.mark.parametrize("name,kw,chunk", [("small_dde", {}, 60000), ("lofar", dict(T=640, nr_stations=6), 300000),
-                                           ("small_dde", dict(C=7, C_block=3), 40000)])
+                                           ("small_dde", dict(C=7, C_block=3), 40000),
+                                           ("small_dde", dict(w_planes=3), 60000)])
 def test_host_streamed_calls(name, kw, chunk, monkeypatch):
     """idg_grid_host / idg_degrid_host (work groups through triple-buffered staging) give the
     device-resident results: degridding bit-identical, gridding equal up to atomic summation order."""
