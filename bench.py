@@ -444,7 +444,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-baseline-s", type=float, default=15.0)
     ap.add_argument("--reference-step-s", type=float, default=8.0)
-    ap.add_argument("--rho-iterations", type=int, default=2048)
+    ap.add_argument("--rho-iterations", type=int, default=16384)
     ap.add_argument("--rho-sweep", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
