@@ -59,7 +59,17 @@ __global__ void loop(float *out, int iters) {
                 else { ah[i][j] = __float_as_uint(cs[j]); al[i][j] = __float_as_uint(sn[j]); }
             }
         }
-        if ((MODE & 4) && (MODE & 8)) {
+        if (MODE & 16) {   // tcgen05-style: stage the split A operands in shared memory (2 x STS.128 / tile)
+            __shared__ uint4 stage[2][64][32];
+            const int slot = it & 1;
+#pragma unroll
+            for (int i = 0; i < MT; ++i) {
+                stage[slot][(threadIdx.x >> 5) * MT + i][lane] = make_uint4(ah[i][0], ah[i][1], ah[i][2], ah[i][3]);
+                stage[slot][(threadIdx.x >> 5) * MT + i + 32][lane] = make_uint4(al[i][0], al[i][1], al[i][2], al[i][3]);
+            }
+            if ((it & 7) == 7) __syncwarp();
+            acc[0][0] += 1e-30f * __uint_as_float(stage[slot ^ 1][0][lane].x);
+        } else if ((MODE & 4) && (MODE & 8)) {
 #pragma unroll
             for (int i = 0; i < MT; ++i) mma_bf(acc[i], ah[i], b0, b1);
 #pragma unroll
@@ -99,14 +109,10 @@ int main() {
     float *out; cudaMalloc(&out, 148 * 64 * 1024 * 4);
     for (int bps : {2, 3}) {
         run<3, 7>("f16 full (sincos+split+mma)", 12, bps, out);
-        run<3, 15>("bf16 full (sincos+PRMT split+mma)", 12, bps, out);
-        run<3, 14>("bf16 split+mma, no sincos", 12, bps, out);
-        run<3, 6>("f16 split+mma, no sincos", 12, bps, out);
-        run<3, 10>("bf16 split, no sincos/mma", 12, bps, out);
-        run<3, 2>("f16 split, no sincos/mma", 12, bps, out);
+        run<3, 3 + 16>("sincos+split+STS (tcgen05 A staging)", 12, bps, out);
+        run<3, 3>("sincos+split", 12, bps, out);
         run<3, 1>("sincos only", 12, bps, out);
     }
-    run<2, 15>("bf16 full MT2 W8", 8, 4, out);
-    run<4, 15>("bf16 full MT4 W9", 9, 3, out);
+    run<4, 3 + 16>("sincos+split+STS MT4 W8", 8, 4, out);
     printf("%s\n", cudaGetErrorString(cudaGetLastError()));
 }
