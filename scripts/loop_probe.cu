@@ -60,12 +60,12 @@ __global__ void loop(float *out, int iters) {
             }
         }
         if (MODE & 16) {   // tcgen05-style: stage the split A operands in shared memory (2 x STS.128 / tile)
-            __shared__ uint4 stage[2][64][32];
+            __shared__ uint4 stage[2][48][32];
             const int slot = it & 1;
 #pragma unroll
             for (int i = 0; i < MT; ++i) {
-                stage[slot][(threadIdx.x >> 5) * MT + i][lane] = make_uint4(ah[i][0], ah[i][1], ah[i][2], ah[i][3]);
-                stage[slot][(threadIdx.x >> 5) * MT + i + 32][lane] = make_uint4(al[i][0], al[i][1], al[i][2], al[i][3]);
+                stage[slot][((threadIdx.x >> 5) * MT + i) % 24][lane] = make_uint4(ah[i][0], ah[i][1], ah[i][2], ah[i][3]);
+                stage[slot][((threadIdx.x >> 5) * MT + i) % 24 + 24][lane] = make_uint4(al[i][0], al[i][1], al[i][2], al[i][3]);
             }
             if ((it & 7) == 7) __syncwarp();
             acc[0][0] += 1e-30f * __uint_as_float(stage[slot ^ 1][0][lane].x);
