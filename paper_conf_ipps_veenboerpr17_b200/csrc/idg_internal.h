@@ -66,6 +66,7 @@ struct Variant {
 const Variant *tc_gridder_variants(int *n);     // split-f16 mma (idg_kernels_tc.cu)
 const Variant *tc_degridder_variants(int *n);
 const Variant *tf32_gridder_variants(int *n);   // split-tf32 mma (idg_kernels_tf32.cu)
+const Variant *umma_gridder_variants(int *n);   // tcgen05 / TMEM (idg_kernels_umma.cu)
 const Variant *tf32_degridder_variants(int *n);
 
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s);

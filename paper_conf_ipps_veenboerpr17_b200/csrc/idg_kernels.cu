@@ -361,6 +361,8 @@ const std::vector<const Variant *> &tensor_variants(int which) {
             for (int i = 0; i < n; ++i) v.push_back(&t[i]);
             t = tf32_gridder_variants(&n);
             for (int i = 0; i < n; ++i) v.push_back(&t[i]);
+            t = umma_gridder_variants(&n);
+            for (int i = 0; i < n; ++i) v.push_back(&t[i]);
             return v;
         }(),
         [] {
