@@ -129,10 +129,10 @@ __device__ __forceinline__ float4 abs_max4(float4 v, float m) {
 // Tensor-core gridder.  One CTA per work item; WARPS warps x MT m-tiles x 16 pixels = N~^2.
 // k-block = 8 visibilities = 8 consecutive channels of one timestep (requires C~ % 8 == 0).
 // ------------------------------------------------------------------------------------------------
-constexpr int kTcBatchKB = 64;  // k-blocks per shared-memory batch (512 visibilities)
+constexpr int kTcBatchKB = 64;  // default k-blocks per shared-memory batch (512 visibilities)
 
-inline size_t gridder_tc_smem_bytes(int NS, int max_channels) {
-    const size_t kbb = kTcBatchKB;
+inline size_t gridder_tc_smem_bytes(int NS, int max_channels, int kbb_ = kTcBatchKB) {
+    const size_t kbb = kbb_;
     const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + kbb * 4 * 16 /*df*/ +
                         (kbb + 1) * 32 /*coef*/ + size_t(max_channels) * 4;
     const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2);
@@ -142,13 +142,13 @@ inline size_t gridder_tc_smem_bytes(int NS, int max_channels) {
 // REC = 1: channels are uniformly spaced, so the phasor of k-slot q+4 (channel c+4) is the phasor of
 // slot q times the per-(pixel, timestep) step exp(i 4 dnu/c Q_t): half of the sincos become one complex
 // multiply (4 FMA-pipe instructions) and the MUFU (XU) load per pair drops from 2 to ~1.25 (+ steps).
-template <int NS, int WARPS, int MT, int MINB, int REC>
+template <int NS, int WARPS, int MT, int MINB, int REC, int KBB_ = kTcBatchKB>
 __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const KernelArgs a) {
     constexpr int NT = WARPS * 32;
     constexpr int NPIX = NS * NS;
     static_assert(WARPS * MT * 16 == NPIX, "warps x m-tiles x 16 must cover the subgrid");
     constexpr int h = NS / 2;
-    constexpr int KBB = kTcBatchKB;
+    constexpr int KBB = KBB_;
     constexpr int VB = KBB * 8;
     extern __shared__ __align__(16) unsigned char smem[];
     float4 *raw_s = reinterpret_cast<float4 *>(smem);                // [VB][2]
@@ -478,13 +478,13 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     }
 }
 
-template <int NS, int WARPS, int MT, int MINB, int REC>
+template <int NS, int WARPS, int MT, int MINB, int REC, int KBB = kTcBatchKB>
 cudaError_t launch_gridder_tc(const KernelArgs &a, cudaStream_t st) {
-    const size_t smem = gridder_tc_smem_bytes(NS, a.max_channels_in_item);
-    cudaError_t err = dev::prepare(gridder_tc_kernel<NS, WARPS, MT, MINB, REC>, smem);
+    const size_t smem = gridder_tc_smem_bytes(NS, a.max_channels_in_item, KBB);
+    cudaError_t err = dev::prepare(gridder_tc_kernel<NS, WARPS, MT, MINB, REC, KBB>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("gridder", st);
-    gridder_tc_kernel<NS, WARPS, MT, MINB, REC><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    gridder_tc_kernel<NS, WARPS, MT, MINB, REC, KBB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -500,6 +500,8 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 
 #define TG(NS, W, MT, MB) \
     {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB, 0>}
+#define TGB(NS, W, MT, MB, KB) \
+    {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KB" #KB ">", launch_gridder_tc<NS, W, MT, MB, 0, KB>}
 #define TGR(NS, W, MT, MB) \
     {NS, 8, kTensor, 1, "gridder_tcr<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB, 1>}
 // First eligible entry is the default.  B200 sweep (LOFAR, SKA-T1024): the direct kernel and the
@@ -514,7 +516,9 @@ const Variant kTcGridder[] = {
     TG(16, 4, 4, 4), TG(16, 8, 2, 3), TG(16, 16, 1, 2),
     TGR(24, 12, 3, 2), TGR(24, 9, 4, 3), TGR(24, 6, 6, 2), TGR(24, 4, 9, 4), TGR(24, 12, 3, 1),
     TGR(16, 4, 4, 4), TGR(16, 8, 2, 3),
+    TGB(24, 12, 3, 2, 128), TGB(24, 12, 3, 2, 32), TGB(24, 12, 3, 2, 256), TGB(32, 16, 4, 2, 128), TGB(32, 16, 4, 2, 32),
 };
+#undef TGB
 #undef TGR
 #undef TG
 #define TD(NS, W, MT, MB) \
