@@ -498,10 +498,10 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-#define TG(NS, W, MT, MB) \
-    {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB, 0>}
 #define TGB(NS, W, MT, MB, KB) \
     {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KB" #KB ">", launch_gridder_tc<NS, W, MT, MB, 0, KB>}
+#define TG(NS, W, MT, MB) \
+    {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB, 0>}
 #define TGR(NS, W, MT, MB) \
     {NS, 8, kTensor, 1, "gridder_tcr<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB, 1>}
 // First eligible entry is the default.  B200 sweep (LOFAR, SKA-T1024): the direct kernel and the
@@ -509,14 +509,14 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 // XU limit), so the direct kernel (no recurrence error) is the default for N~ = 24; for N~ = 32 the
 // recurrence variant is 1% faster.
 const Variant kTcGridder[] = {
-    TG(24, 12, 3, 2), TG(24, 6, 6, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
+    TGB(24, 12, 3, 2, 128), TG(24, 12, 3, 2), TG(24, 6, 6, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
     TG(24, 6, 6, 3), TG(24, 9, 4, 3), TG(24, 4, 9, 4),
     TGR(32, 8, 8, 2), TGR(32, 16, 4, 2), TGR(32, 16, 4, 1),
     TG(32, 16, 4, 2), TG(32, 8, 8, 2), TG(32, 16, 4, 1), TG(32, 4, 16, 3), TG(32, 8, 8, 3),
     TG(16, 4, 4, 4), TG(16, 8, 2, 3), TG(16, 16, 1, 2),
     TGR(24, 12, 3, 2), TGR(24, 9, 4, 3), TGR(24, 6, 6, 2), TGR(24, 4, 9, 4), TGR(24, 12, 3, 1),
     TGR(16, 4, 4, 4), TGR(16, 8, 2, 3),
-    TGB(24, 12, 3, 2, 128), TGB(24, 12, 3, 2, 32), TGB(24, 12, 3, 2, 256), TGB(32, 16, 4, 2, 128), TGB(32, 16, 4, 2, 32),
+    TGB(24, 12, 3, 2, 32), TGB(24, 12, 3, 2, 256), TGB(32, 16, 4, 2, 128), TGB(32, 16, 4, 2, 32),
 };
 #undef TGB
 #undef TGR
