@@ -105,14 +105,63 @@ void run(const char *name, int warps, int bps, float *out) {
     int clk; cudaDeviceGetAttribute(&clk, cudaDevAttrClockRate, 0);
     printf("%-34s warps/SM %3d: %6.2f pairs/clk/SM\n", name, warps * bps, pairs / (ms * 1e-3) / 148 / 1.965e9);
 }
+
+// software-pipelined variant: sincos of iteration it+1 are issued before the split + mma of iteration it
+template <int MT>
+__global__ void loop_pipe(float *out, int iters) {
+    const int lane = threadIdx.x & 31;
+    u64 B[MT], Q[MT];
+    float acc[MT][4];
+    for (int i = 0; i < MT; ++i) { B[i] = pk(0.1f * i + lane * 1e-3f, 0.2f); Q[i] = pk(0.3f, 0.4f + i * 1e-2f); for (int j = 0; j < 4; ++j) acc[i][j] = 0; }
+    uint32_t b0 = 0x3c003c00u ^ lane, b1 = 0x3c003c01u, b2 = 0x3c013c00u, b3 = lane;
+    u64 dq = pk(1e-3f, 2e-3f), dq4 = pk(3e-3f, 4e-3f);
+    float sn[MT][4], cs[MT][4];
+    auto phasors = [&](float (&sn_)[MT][4], float (&cs_)[MT][4]) {
+        dq = fma2(dq, pk(1.0000001f, 1.0000001f), pk(1e-7f, 1e-7f));
+        dq4 = fma2(dq4, pk(1.0000001f, 1.0000001f), pk(2e-7f, 2e-7f));
+#pragma unroll
+        for (int i = 0; i < MT; ++i) {
+            float2 p0 = up(fma2(dq, Q[i], B[i])), p1 = up(fma2(dq4, Q[i], B[i]));
+            __sincosf(p0.x, &sn_[i][0], &cs_[i][0]); __sincosf(p0.y, &sn_[i][1], &cs_[i][1]);
+            __sincosf(p1.x, &sn_[i][2], &cs_[i][2]); __sincosf(p1.y, &sn_[i][3], &cs_[i][3]);
+        }
+    };
+    phasors(sn, cs);
+    for (int it = 0; it < iters; ++it) {
+        uint32_t ah[MT][4], al[MT][4];
+#pragma unroll
+        for (int i = 0; i < MT; ++i)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) split(cs[i][j], sn[i][j], ah[i][j], al[i][j]);
+        phasors(sn, cs);   // next iteration's MUFU work, independent of the mma below
+#pragma unroll
+        for (int i = 0; i < MT; ++i) mma(acc[i], ah[i], b0, b1);
+#pragma unroll
+        for (int i = 0; i < MT; ++i) mma(acc[i], ah[i], b2, b3);
+#pragma unroll
+        for (int i = 0; i < MT; ++i) mma(acc[i], al[i], b0, b1);
+    }
+    float s = 0; for (int i = 0; i < MT; ++i) for (int j = 0; j < 4; ++j) s += acc[i][j];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+template <int MT>
+void run_pipe(const char *name, int warps, int bps, float *out) {
+    const int iters = 2048;
+    const int blocks = 148 * bps, threads = 32 * warps;
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    loop_pipe<MT><<<blocks, threads>>>(out, 16); cudaDeviceSynchronize();
+    cudaEventRecord(e0); loop_pipe<MT><<<blocks, threads>>>(out, iters); cudaEventRecord(e1); cudaEventSynchronize(e1);
+    float ms; cudaEventElapsedTime(&ms, e0, e1);
+    double pairs = double(blocks) * threads * iters * MT * 4;
+    printf("%-34s warps/SM %3d: %6.2f pairs/clk/SM\n", name, warps * bps, pairs / (ms * 1e-3) / 148 / 1.965e9);
+}
 int main() {
     float *out; cudaMalloc(&out, 148 * 64 * 1024 * 4);
-    for (int bps : {2, 3}) {
+    for (int bps : {1, 2, 3}) {
         run<3, 7>("f16 full (sincos+split+mma)", 12, bps, out);
-        run<3, 3 + 16>("sincos+split+STS (tcgen05 A staging)", 12, bps, out);
-        run<3, 3>("sincos+split", 12, bps, out);
-        run<3, 1>("sincos only", 12, bps, out);
+        run_pipe<3>("pipelined full MT3 W12", 12, bps, out);
     }
-    run<4, 3 + 16>("sincos+split+STS MT4 W8", 8, 4, out);
+    run_pipe<2>("pipelined full MT2 W8", 8, 4, out);
+    run_pipe<4>("pipelined full MT4 W8", 8, 3, out);
     printf("%s\n", cudaGetErrorString(cudaGetLastError()));
 }
