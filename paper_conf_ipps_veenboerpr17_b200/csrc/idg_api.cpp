@@ -78,6 +78,7 @@ struct idg_plan {
     std::vector<int32_t> order;      // launch order: largest T~ C~ first (tail balance)
     int64_t nr_vis_assigned = 0, nr_vis_dropped = 0, nr_pairs = 0;
     int32_t max_channels_in_item = 0;
+    int32_t max_timesteps_in_item = 0;
     std::vector<WorkGroup> groups;   // host-streamed work groups
     size_t group_bytes = 0;          // largest work group's visibility bytes
     int32_t channel_gcd = 1;
@@ -261,6 +262,7 @@ idg::KernelArgs make_args(const idg_plan *plan, const DeviceCopy *dc, const floa
     a.vis = static_cast<float2 *>(d_vis);
     a.grid = static_cast<float2 *>(d_grid);
     a.max_channels_in_item = plan->max_channels_in_item;
+    a.max_timesteps_in_item = plan->max_timesteps_in_item;
     a.channel_gcd = plan->channel_gcd;
     a.channels_uniform = plan->channels_uniform;
     a.channel_step = plan->channel_step;
@@ -346,6 +348,7 @@ idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, i
             const int nc = it.channel_end - it.channel_begin;
             plan->nr_pairs += npix * it.nr_timesteps * nc;
             plan->max_channels_in_item = std::max(plan->max_channels_in_item, nc);
+            plan->max_timesteps_in_item = std::max(plan->max_timesteps_in_item, it.nr_timesteps);
             g = std::gcd(g, nc);
         }
         plan->channel_gcd = g == 0 ? 1 : g;

@@ -47,6 +47,7 @@ struct KernelArgs {
     float2 *vis;                 // [nbl][T][C][4]  (const for gridding)
     float2 *grid;                // [4][N][N]       (const for degridding)
     int32_t max_channels_in_item;
+    int32_t max_timesteps_in_item;
     int32_t channel_gcd;         // gcd of all items' channel counts
     int32_t channels_uniform;    // 1 if nu_{c+1} - nu_c is the same for all c (to 1e-9 relative)
     float channel_step;          // (nu_{c+1} - nu_c) / c  [1/m], valid when channels_uniform

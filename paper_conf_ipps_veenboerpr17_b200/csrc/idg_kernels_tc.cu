@@ -338,9 +338,10 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
 // B fragments (k-block = 8 pixels) + per-pixel {l, m, n}; m-tile = 16 consecutive visibilities of
 // the item (flattened (t, c) order); each warp takes MT tiles at a time over all k-blocks.
 // ------------------------------------------------------------------------------------------------
-inline size_t degridder_tc_smem_bytes(int NS) {
+inline size_t degridder_tc_smem_bytes(int NS, int max_timesteps, int max_channels) {
     const size_t npix = size_t(NS) * NS;
-    return npix * 64 /*sub+tmp | frag*/ + npix * 4 * 8 / 2 /*lmn slot pairs: 32 B per 2 pixels*/ + 16;
+    return npix * 64 /*sub+tmp | frag*/ + npix * 4 * 8 / 2 /*lmn slot pairs: 32 B per 2 pixels*/ +
+           size_t(max_timesteps) * 16 /*uvw of the item's timesteps*/ + size_t(max_channels) * 8 /*nu/c*/ + 16;
 }
 
 template <int NS, int WARPS, int MT, int MINB>
@@ -356,6 +357,8 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     float2 *tmp_s = sub_s + 4 * NPIX;                                     // [4][NS][NS]
     uint4 *frag_s = reinterpret_cast<uint4 *>(smem);                      // [NKB][32] (after prologue)
     float4 *lmn_s = reinterpret_cast<float4 *>(smem + size_t(NPIX) * 64); // [NKB][4][2] slot pairs
+    float4 *uvw_s = lmn_s + NKB * 8;                                      // [T~]: u, v, w of the item
+    double *fq_s = reinterpret_cast<double *>(uvw_s + a.max_timesteps_in_item);  // [C~]: nu / c
     __shared__ float red_s[WARPS];
     __shared__ float2 tw[NS];
 
@@ -365,7 +368,14 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     const int nc = s.nc;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
 
-    dev::degridder_split_columns<NS>(a, s, sub_s, tmp_s, tw);
+    // the item's uvw and nu/c, read by every tile's phase coefficients (staged once: no dependent
+    // global loads in front of each tile's k-block loop)
+    for (int t = threadIdx.x; t < md.nr_timesteps; t += NT) {
+        const float *p = a.uvw + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset + t) * 3;
+        uvw_s[t] = make_float4(p[0], p[1], p[2], 0.0f);
+    }
+    for (int c = threadIdx.x; c < nc; c += NT) fq_s[c] = a.frequencies[md.channel_begin + c] / kSpeedOfLight;
+    dev::degridder_split_columns<NS>(a, s, sub_s, tmp_s, tw);  // (its barriers publish uvw_s / fq_s)
     float2 rr[PPT][4];
     float mx = 0.0f;
 #pragma unroll
@@ -425,11 +435,11 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
                 float fu = 0.0f, fv = 0.0f, fw = 0.0f;
                 if (v < nvis) {
                     const int t = v / nc, c = v - t * nc;
-                    const float *p = a.uvw + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset + t) * 3;
-                    const double f = a.frequencies[md.channel_begin + c] / kSpeedOfLight;
-                    fu = float(dev::kTwoPi * (double(p[0]) * f - s.u0));
-                    fv = float(dev::kTwoPi * (double(p[1]) * f - s.v0));
-                    fw = float(dev::kTwoPi * (double(p[2]) * f - s.w0));
+                    const float4 p = uvw_s[t];
+                    const double f = fq_s[c];
+                    fu = float(dev::kTwoPi * (double(p.x) * f - s.u0));
+                    fv = float(dev::kTwoPi * (double(p.y) * f - s.v0));
+                    fw = float(dev::kTwoPi * (double(p.z) * f - s.w0));
                 }
                 cu[i][r] = dup(fu);
                 cv[i][r] = dup(fv);
@@ -490,7 +500,7 @@ cudaError_t launch_gridder_tc(const KernelArgs &a, cudaStream_t st) {
 
 template <int NS, int WARPS, int MT, int MINB>
 cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
-    const size_t smem = degridder_tc_smem_bytes(NS);
+    const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
     cudaError_t err = dev::prepare(degridder_tc_kernel<NS, WARPS, MT, MINB>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("degridder", st);

@@ -31,6 +31,31 @@ __device__ __forceinline__ void mma(float (&d)[4], const uint32_t (&a)[4], uint3
     asm("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3},{%4,%5,%6,%7},{%8,%9},{%0,%1,%2,%3};"
         : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3]) : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
 }
+
+__device__ __forceinline__ u64 add2(u64 a, u64 b) { u64 r; asm("add.rn.f32x2 %0,%1,%2;" : "=l"(r) : "l"(a), "l"(b)); return r; }
+__device__ __forceinline__ u64 mul2(u64 a, u64 b) { u64 r; asm("mul.rn.f32x2 %0,%1,%2;" : "=l"(r) : "l"(a), "l"(b)); return r; }
+// sincos on the FMA pipe, two arguments packed: exact reduction to r in [-1/2, 1/2] turns, minimax
+// sin(pi r) = r P(r^2), cos(pi r) = Q(r^2), double angle.  |err| <= 7.3e-7.
+__device__ __forceinline__ void poly_sincos2(u64 x, u64 &sn, u64 &cs) {
+    const u64 M = pk(12582912.0f, 12582912.0f);
+    u64 r = mul2(x, pk(0.15915494309189535f, 0.15915494309189535f));
+    const u64 k = sub2(add2(r, M), M);
+    r = sub2(r, k);
+    const u64 t = mul2(r, r);
+    u64 ps = fma2(pk(0.07755820453166962f, 0.07755820453166962f), t, pk(-0.5982410311698914f, -0.5982410311698914f));
+    ps = fma2(ps, t, pk(2.550069570541382f, 2.550069570541382f));
+    ps = fma2(ps, t, pk(-5.167709827423096f, -5.167709827423096f));
+    ps = fma2(ps, t, pk(3.1415927410125732f, 3.1415927410125732f));
+    ps = mul2(ps, r);
+    u64 pc = fma2(pk(0.21968808770179749f, 0.21968808770179749f), t, pk(-1.3318758010864258f, -1.3318758010864258f));
+    pc = fma2(pc, t, pk(4.058411121368408f, 4.058411121368408f));
+    pc = fma2(pc, t, pk(-4.934792995452881f, -4.934792995452881f));
+    pc = fma2(pc, t, pk(0.9999999403953552f, 0.9999999403953552f));
+    const u64 u = add2(ps, ps);
+    sn = mul2(u, pc);
+    const float2 uu = up(u);
+    cs = fma2(pk(-uu.x, -uu.y), ps, pk(1.0f, 1.0f));
+}
 // MODE bits: 1 = sincos, 2 = split, 4 = mma
 template <int MT, int MODE>
 __global__ void loop(float *out, int iters) {
@@ -50,7 +75,14 @@ __global__ void loop(float *out, int iters) {
             float ph[4] = {p0.x, p0.y, p1.x, p1.y}, sn[4], cs[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
+                if ((MODE & 32) && j >= 2) continue;
                 if (MODE & 1) __sincosf(ph[j], &sn[j], &cs[j]); else { sn[j] = ph[j] * 0.5f; cs[j] = ph[j] + 0.25f; }
+            }
+            if (MODE & 32) {   // slots 2, 3 on the FMA pipe (50% of the phasors)
+                u64 s2, c2;
+                poly_sincos2(pk(p1.x, p1.y), s2, c2);
+                const float2 a = up(s2), b = up(c2);
+                sn[2] = a.x; sn[3] = a.y; cs[2] = b.x; cs[3] = b.y;
             }
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
@@ -157,11 +189,11 @@ void run_pipe(const char *name, int warps, int bps, float *out) {
 }
 int main() {
     float *out; cudaMalloc(&out, 148 * 64 * 1024 * 4);
-    for (int bps : {1, 2, 3}) {
+    for (int bps : {2, 3}) {
         run<3, 7>("f16 full (sincos+split+mma)", 12, bps, out);
-        run_pipe<3>("pipelined full MT3 W12", 12, bps, out);
+        run<3, 7 | 32>("full, 50% sincos as FMA poly", 12, bps, out);
+        run<3, 1 | 32>("sincos only, 50% FMA poly", 12, bps, out);
     }
-    run_pipe<2>("pipelined full MT2 W8", 8, 4, out);
-    run_pipe<4>("pipelined full MT4 W8", 8, 3, out);
+    run<2, 7 | 32>("MT2 full, 50% poly", 8, 4, out);
     printf("%s\n", cudaGetErrorString(cudaGetLastError()));
 }
