@@ -8,6 +8,12 @@ those baselines (tested in tests/test_parallel.py).  The path has one exchange p
               torch.distributed reduce to the destination rank (the adder across ranks, P:73);
   degridding: the model grid is broadcast from the source rank; every rank degrids its own shard.
 
+Both collectives can be restricted to the band of grid rows the items cover ("reduce only
+the uv bounding box of the coverage"): the union over ranks of [min y, max y + N~) is agreed with one
+2-element all-reduce, and each contiguous [plane][pol] row slab is reduced / broadcast on its own.  Rows
+outside the band are zero on every rank after gridding and read by no item when degridding, so the
+result is identical to the full-grid collective with less traffic.
+
 torch.distributed is plumbing only (NCCL over NVLink on B200, gloo for the CPU tests); every step of the
 hot path runs in libidg_b200.so.
 """
@@ -40,49 +46,96 @@ def shard_arrays(uvw: np.ndarray, baselines: np.ndarray, b0: int, b1: int):
     return np.ascontiguousarray(uvw[b0:b1]), np.ascontiguousarray(baselines[b0:b1])
 
 
-def reduce_grid(grid, dst: int = 0, group=None):
-    """Sum the ranks' complex64 uv-grids onto `dst` (in place on dst).  Complex is reduced as fp32 pairs."""
+def coverage_rows(item_y, subgrid_size: int, grid_size: int):
+    """Grid rows [y0, y1) covered by items with corner rows `item_y` (empty: (grid_size, 0))."""
+    y = np.asarray(item_y)
+    if y.size == 0:
+        return grid_size, 0
+    return int(y.min()), int(y.max()) + subgrid_size
+
+
+def union_rows(rows, device=None, group=None):
+    """Union over ranks of the local row bands (one 2-element MAX all-reduce)."""
     import torch
+    import torch.distributed as dist
+    y0, y1 = rows
+    if not dist.is_initialized() or dist.get_world_size(group) == 1:
+        return y0, y1
+    t = torch.tensor([-y0, y1], dtype=torch.int64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return int(-t[0]), int(t[1])
+
+
+def _slabs(grid, rows):
+    """Contiguous [plane][pol] row slabs grid[..., y0:y1, :] as fp32 views (the whole grid if rows is None)."""
+    import torch
+    if rows is None:
+        return [torch.view_as_real(grid)]
+    y0, y1 = rows
+    if y1 <= y0:
+        return []
+    n = grid.shape[-1]
+    planes = grid.reshape(-1, grid.shape[-2], n)
+    return [torch.view_as_real(planes[k, y0:y1]) for k in range(planes.shape[0])]
+
+
+def reduce_grid(grid, dst: int = 0, group=None, rows=None):
+    """Sum the ranks' complex64 uv-grids onto `dst` (in place on dst).  Complex is reduced as fp32 pairs.
+    `rows` = (y0, y1), the same on every rank: reduce only that band of every plane/polarisation."""
     import torch.distributed as dist
     if not dist.is_initialized() or dist.get_world_size(group) == 1:
         return grid
-    dist.reduce(torch.view_as_real(grid), dst=dst, op=dist.ReduceOp.SUM, group=group)
+    for slab in _slabs(grid, rows):
+        dist.reduce(slab, dst=dst, op=dist.ReduceOp.SUM, group=group)
     return grid
 
 
-def broadcast_grid(grid, src: int = 0, group=None):
-    """Broadcast the model grid from `src` to every rank (in place)."""
-    import torch
+def broadcast_grid(grid, src: int = 0, group=None, rows=None):
+    """Broadcast the model grid from `src` to every rank (in place); `rows` as for reduce_grid."""
     import torch.distributed as dist
     if not dist.is_initialized() or dist.get_world_size(group) == 1:
         return grid
-    dist.broadcast(torch.view_as_real(grid), src=src, group=group)
+    for slab in _slabs(grid, rows):
+        dist.broadcast(slab, src=src, group=group)
     return grid
 
 
 class ShardedIDG:
-    """The rank-local plan plus the two collectives.  Inputs are the rank's baseline slice."""
+    """The rank-local plan plus the two collectives.  Inputs are the rank's baseline slice.
+    With `bbox` (default) the collectives move only the union band of covered grid rows."""
 
-    def __init__(self, plan):
+    def __init__(self, plan, bbox: bool = True):
         self.plan = plan
+        self.bbox = bbox
+        self._rows = None
+
+    def rows(self, device=None):
+        """The agreed row band (collective on first use; every rank must call it)."""
+        if not self.bbox:
+            return None
+        if self._rows is None:
+            md = self.plan.metadata()
+            local = coverage_rows(md["y"], self.plan.subgrid_size, self.plan.grid_size)
+            self._rows = union_rows(local, device=device)
+        return self._rows
 
     def grid(self, vis, uvw, aterms, taper, grid_out, dst: int = 0, stream=None):
         from . import idg
         idg.grid(self.plan, vis, uvw, aterms, taper, grid_out, stream=stream)
-        return reduce_grid(grid_out, dst=dst)
+        return reduce_grid(grid_out, dst=dst, rows=self.rows(grid_out.device))
 
     def degrid(self, grid_in, uvw, aterms, taper, vis_out, src: int = 0, stream=None):
         from . import idg
-        broadcast_grid(grid_in, src=src)
+        broadcast_grid(grid_in, src=src, rows=self.rows(grid_in.device))
         return idg.degrid(self.plan, grid_in, uvw, aterms, taper, vis_out, stream=stream)
 
     # host-streamed variants (visibilities in pinned host memory, P:198-212)
     def grid_host(self, vis_host, uvw, aterms, taper, grid_out, ws, dst: int = 0, stream=None):
         from . import idg
         idg.grid_host(self.plan, vis_host, uvw, aterms, taper, grid_out, ws, stream=stream)
-        return reduce_grid(grid_out, dst=dst)
+        return reduce_grid(grid_out, dst=dst, rows=self.rows(grid_out.device))
 
     def degrid_host(self, grid_in, uvw, aterms, taper, vis_host_out, ws, src: int = 0, stream=None):
         from . import idg
-        broadcast_grid(grid_in, src=src)
+        broadcast_grid(grid_in, src=src, rows=self.rows(grid_in.device))
         return idg.degrid_host(self.plan, grid_in, uvw, aterms, taper, vis_host_out, ws, stream=stream)

@@ -58,17 +58,26 @@ def _worker(rank, world, port, result_dir):
     b0, b1 = parallel.shard_range(obs.nr_baselines, rank, world)
     sub = obs.subset(nr_baselines=b1 - b0, baseline_begin=b0)
     items, _ = oracle.plan(sub)
-    # gridding: per-rank grid, then the product's reduce
+    # gridding: per-rank grid, then the product's reduce (full grid, and the covered row band only)
     g = torch.from_numpy(oracle.grid(sub, items, vis[b0:b1], aterms, taper).astype(np.complex64))
+    g_band = g.clone()
+    rows = parallel.union_rows(parallel.coverage_rows(items["y"], obs.subgrid_size, obs.grid_size))
     parallel.reduce_grid(g, dst=0)
+    parallel.reduce_grid(g_band, dst=0, rows=rows)
     # degridding: the model grid exists on rank 0 only, the product's broadcast ships it
     model = torch.from_numpy(idgsynth.make_grid(obs)) if rank == 0 else torch.zeros(
         (4, obs.grid_size, obs.grid_size), dtype=torch.complex64)
+    model_band = model.clone() if rank == 0 else torch.full_like(model, float("nan"))
     parallel.broadcast_grid(model, src=0)
+    parallel.broadcast_grid(model_band, src=0, rows=rows)   # rows outside the band stay NaN off rank 0
     v = oracle.scatter_visibilities(sub, items, oracle.degrid(sub, items, model.numpy(), aterms, taper))
+    v_band = oracle.scatter_visibilities(sub, items, oracle.degrid(sub, items, model_band.numpy(), aterms, taper))
     np.save(os.path.join(result_dir, f"vis{rank}.npy"), v)
+    np.save(os.path.join(result_dir, f"vis_band{rank}.npy"), v_band)
     if rank == 0:
         np.save(os.path.join(result_dir, "grid.npy"), g.numpy())
+        np.save(os.path.join(result_dir, "grid_band.npy"), g_band.numpy())
+        np.save(os.path.join(result_dir, "rows.npy"), np.array(rows))
     dist.destroy_process_group()
 
 
@@ -86,3 +95,19 @@ def test_gloo_two_ranks_compose_to_single_process(tmp_path):
     ref_v = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, idgsynth.make_grid(obs), aterms, taper))
     got_v = np.concatenate([np.load(tmp_path / f"vis{r}.npy") for r in range(world)], axis=0)
     np.testing.assert_allclose(got_v, ref_v, rtol=0, atol=1e-9 * np.abs(ref_v).max())
+    # the row-band collectives give the identical result with a strictly smaller message
+    y0, y1 = np.load(tmp_path / "rows.npy")
+    assert 0 <= y0 < y1 <= obs.grid_size and (y1 - y0) < obs.grid_size
+    np.testing.assert_array_equal(np.load(tmp_path / "grid_band.npy"), got)
+    for r in range(world):
+        np.testing.assert_array_equal(np.load(tmp_path / f"vis_band{r}.npy"), np.load(tmp_path / f"vis{r}.npy"))
+
+
+def test_coverage_rows():
+    assert parallel.coverage_rows(np.array([5, 40, 17]), 24, 128) == (5, 64)
+    assert parallel.coverage_rows(np.array([], dtype=np.int32), 24, 128) == (128, 0)
+    assert parallel.union_rows((5, 64)) == (5, 64)            # single process: identity
+    g = torch.arange(2 * 4 * 6 * 6, dtype=torch.float32).reshape(2, 4, 6, 6).to(torch.complex64)
+    slabs = parallel._slabs(g, (1, 3))
+    assert len(slabs) == 8 and all(s.is_contiguous() and s.shape == (2, 6, 2) for s in slabs)
+    assert parallel._slabs(g, (3, 3)) == []
