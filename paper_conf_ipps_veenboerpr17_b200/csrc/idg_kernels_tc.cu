@@ -63,26 +63,19 @@ __device__ __forceinline__ f2p sub2(f2p a, f2p b) {
 }
 
 // (x, y) -> f16x2 hi = rn(x, y) and lo = rn(x - hi, y - hi): x = hi + lo to ~22 significant bits.
-// Used for the B operands (once per batch / item).
+// x - hi is one mixed-precision FHFMA per value (fma.rn.f32.f16: hi * -1 + x, f16 operands, f32 result;
+// exact, since hi is x rounded), so a split is F2FP + 2 FHFMA + F2FP.  Used for the phasors (per pair, on
+// the critical path) and for the B operands (once per batch / item).  For |x| < 2^-14 (f16 subnormal)
+// the residual error is below 2^-25.
 __device__ __forceinline__ void split2(float x, float y, uint32_t &hi, uint32_t &lo) {
-    const __half2 h = __floats2half2_rn(x, y);
-    const float2 hf = __half22float2(h);
-    const float2 d = unpk(sub2(pk(x, y), pk(hf.x, hf.y)));  // one FADD2 for both residuals
-    const __half2 l = __floats2half2_rn(d.x, d.y);
-    hi = h2_bits(h);
-    lo = h2_bits(l);
+    hi = h2_bits(__floats2half2_rn(x, y));
+    float dx, dy;
+    asm("{\n.reg .f16 a, b, m;\nmov.b32 {a, b}, %2;\nmov.b16 m, 0xBC00;\n"
+        "fma.rn.f32.f16 %0, a, m, %3;\nfma.rn.f32.f16 %1, b, m, %4;\n}"
+        : "=f"(dx), "=f"(dy) : "r"(hi), "f"(x), "f"(y));
+    lo = h2_bits(__floats2half2_rn(dx, dy));
 }
-
-// Phasor split (|x|, |y| <= 1, per pair, on the critical path): hi = x with the low 13 mantissa bits
-// cleared (LOP3 on the ALU pipe; exactly representable in f16 for |x| >= 2^-14, and within 2^-25
-// otherwise), lo = x - hi (one FADD2, exact) -> f16.  |lo| < 2^-10 |x|, so x = hi + lo to ~21 bits.
-__device__ __forceinline__ void split_phasor(float x, float y, uint32_t &hi, uint32_t &lo) {
-    const float hx = __uint_as_float(__float_as_uint(x) & 0xffffe000u);
-    const float hy = __uint_as_float(__float_as_uint(y) & 0xffffe000u);
-    const float2 d = unpk(sub2(pk(x, y), pk(hx, hy)));
-    hi = h2_bits(__floats2half2_rn(hx, hy));
-    lo = h2_bits(__floats2half2_rn(d.x, d.y));
-}
+__device__ __forceinline__ void split_phasor(float x, float y, uint32_t &hi, uint32_t &lo) { split2(x, y, hi, lo); }
 
 __device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
                                          uint32_t b0, uint32_t b1) {

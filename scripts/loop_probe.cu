@@ -17,6 +17,16 @@ __device__ __forceinline__ void split(float x, float y, uint32_t &hi, uint32_t &
     hi = h2b(__floats2half2_rn(hx, hy)); lo = h2b(__floats2half2_rn(d.x, d.y));
 }
 // bf16 split without conversions: hi = upper halves (PRMT), lo = x - hi (FADD2), truncated by PRMT
+// hi = rn_f16(x, y); lo = rn_f16(x - hi, y - hi) with the mixed-precision FHFMA (f16 * f16 + f32)
+__device__ __forceinline__ void split_mx(float x, float y, uint32_t &hi, uint32_t &lo) {
+    const __half2 h = __floats2half2_rn(x, y);
+    hi = h2b(h);
+    float lx, ly;
+    asm("{\n.reg .f16 a, b, m;\nmov.b32 {a, b}, %2;\nmov.b16 m, 0xBC00;\n"
+        "fma.rn.f32.f16 %0, a, m, %3;\nfma.rn.f32.f16 %1, b, m, %4;\n}"
+        : "=f"(lx), "=f"(ly) : "r"(hi), "f"(x), "f"(y));
+    lo = h2b(__floats2half2_rn(lx, ly));
+}
 __device__ __forceinline__ void split_bf(float x, float y, uint32_t &hi, uint32_t &lo) {
     hi = __byte_perm(__float_as_uint(x), __float_as_uint(y), 0x7632);
     float hx = __uint_as_float(__float_as_uint(x) & 0xffff0000u), hy = __uint_as_float(__float_as_uint(y) & 0xffff0000u);
@@ -86,7 +96,8 @@ __global__ void loop(float *out, int iters) {
             }
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
-                if (MODE & 8) split_bf(cs[j], sn[j], ah[i][j], al[i][j]);
+                if (MODE & 64) split_mx(cs[j], sn[j], ah[i][j], al[i][j]);
+                else if (MODE & 8) split_bf(cs[j], sn[j], ah[i][j], al[i][j]);
                 else if (MODE & 2) split(cs[j], sn[j], ah[i][j], al[i][j]);
                 else { ah[i][j] = __float_as_uint(cs[j]); al[i][j] = __float_as_uint(sn[j]); }
             }
@@ -191,9 +202,9 @@ int main() {
     float *out; cudaMalloc(&out, 148 * 64 * 1024 * 4);
     for (int bps : {2, 3}) {
         run<3, 7>("f16 full (sincos+split+mma)", 12, bps, out);
-        run<3, 7 | 32>("full, 50% sincos as FMA poly", 12, bps, out);
-        run<3, 1 | 32>("sincos only, 50% FMA poly", 12, bps, out);
+        run<3, 7 | 64>("full, FHFMA split", 12, bps, out);
+        run<3, 6 | 64>("FHFMA split + mma only", 12, bps, out);
+        run<3, 6>("LOP3 split + mma only", 12, bps, out);
     }
-    run<2, 7 | 32>("MT2 full, 50% poly", 8, 4, out);
     printf("%s\n", cudaGetErrorString(cudaGetLastError()));
 }
