@@ -89,6 +89,7 @@ def main():
     ap.add_argument("--config", default="lofar")
     ap.add_argument("--launches")
     ap.add_argument("--note", default="")
+    ap.add_argument("--bench", help="bench.py JSON line of the same build: adds its CUDA-event shares")
     args = ap.parse_args()
     md = [f"# ncu summary {args.tag} ({args.config})", ""]
     if args.note:
@@ -109,8 +110,19 @@ def main():
     if args.launches:
         md += ["## launch list (ncu gpu__time_duration, cold/serialised: compare shares)", "",
                "| kernel | launches | total ms | share |", "|---|---|---|---|"]
-        for k, n, ms, sh in launches(args.launches):
+        rows = launches(args.launches)
+        for k, n, ms, sh in rows:
             md.append(f"| `{k}` | {n} | {ms:.3f} | {sh:.1f}% |")
+        # the timed step = grid zeroing + gridder + degridder; the rho benchmarks run after it
+        step = [(k, n, ms) for k, n, ms, _ in rows if "gridder" in k or "FillFunctor" in k]
+        tot = sum(ms / n for _, n, ms in step)
+        bench = json.load(open(args.bench)).get("kernels", {}) if args.bench else {}
+        md += ["", "Share of the timed step (fill + gridder + degridder), ncu launch list vs bench.py CUDA events:", "",
+               "| kernel | mean ms / launch (ncu) | share (ncu) | share (bench) |", "|---|---|---|---|"]
+        for k, n, ms in step:
+            short = "degridder" if "degridder" in k else "gridder" if "gridder" in k else None
+            b = bench.get(short, {}).get("share_of_step") if short else None
+            md.append(f"| `{k}` | {ms / n:.3f} | {ms / n / tot:.4f} | {'-' if b is None else f'{b:.4f}'} |")
     open(os.path.join(ROOT, "profiles", f"{args.tag}_ncu_summary.md"), "w").write("\n".join(md) + "\n")
     json.dump(js, open(js_path, "w"), indent=1)
 
