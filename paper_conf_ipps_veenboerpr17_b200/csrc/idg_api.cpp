@@ -128,36 +128,44 @@ struct idg_plan {
                                                  prop.name + " is sm_" + std::to_string(prop.major) +
                                                  std::to_string(prop.minor));
         DeviceCopy dc;
+        auto release = [&dc]() {  // undo a partial device copy
+            cudaFree(dc.items); cudaFree(dc.order); cudaFree(dc.iota); cudaFree(dc.baselines);
+            cudaFree(dc.frequencies);
+            if (dc.h2d) cudaStreamDestroy(dc.h2d);
+            if (dc.d2h) cudaStreamDestroy(dc.d2h);
+        };
         const size_t ni = std::max<size_t>(1, items.size());
         if ((e = cudaMalloc(&dc.items, ni * sizeof(idg_metadata))) != cudaSuccess ||
             (e = cudaMalloc(&dc.order, ni * sizeof(int32_t))) != cudaSuccess ||
             (e = cudaMalloc(&dc.iota, ni * sizeof(int32_t))) != cudaSuccess ||
             (e = cudaMalloc(&dc.baselines, std::max<size_t>(2, baselines.size()) * 4)) != cudaSuccess ||
             (e = cudaMalloc(&dc.frequencies, frequencies.size() * 8)) != cudaSuccess) {
-            cudaFree(dc.items); cudaFree(dc.order); cudaFree(dc.iota); cudaFree(dc.baselines);
-            cudaFree(dc.frequencies);
+            release();
             return e == cudaErrorMemoryAllocation ? fail(IDG_ERR_OUT_OF_MEMORY, "plan device copy")
                                                   : cuda_fail(e, "cudaMalloc(plan)");
         }
-        if (!items.empty()) {
-            cudaMemcpy(dc.items, items.data(), items.size() * sizeof(idg_metadata), cudaMemcpyHostToDevice);
-            cudaMemcpy(dc.order, order.data(), order.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
-            std::vector<int32_t> iota(items.size());
-            std::iota(iota.begin(), iota.end(), 0);
-            cudaMemcpy(dc.iota, iota.data(), iota.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
+        std::vector<int32_t> iota(items.size());
+        std::iota(iota.begin(), iota.end(), 0);
+        if ((!items.empty() &&
+             ((e = cudaMemcpy(dc.items, items.data(), items.size() * sizeof(idg_metadata), cudaMemcpyHostToDevice)) != cudaSuccess ||
+              (e = cudaMemcpy(dc.order, order.data(), order.size() * sizeof(int32_t), cudaMemcpyHostToDevice)) != cudaSuccess ||
+              (e = cudaMemcpy(dc.iota, iota.data(), iota.size() * sizeof(int32_t), cudaMemcpyHostToDevice)) != cudaSuccess)) ||
+            (!baselines.empty() &&
+             (e = cudaMemcpy(dc.baselines, baselines.data(), baselines.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess) ||
+            (e = cudaMemcpy(dc.frequencies, frequencies.data(), frequencies.size() * 8, cudaMemcpyHostToDevice)) != cudaSuccess) {
+            release();
+            return cuda_fail(e, "cudaMemcpy(plan)");
         }
         if ((e = cudaStreamCreateWithFlags(&dc.h2d, cudaStreamNonBlocking)) != cudaSuccess ||
-            (e = cudaStreamCreateWithFlags(&dc.d2h, cudaStreamNonBlocking)) != cudaSuccess)
+            (e = cudaStreamCreateWithFlags(&dc.d2h, cudaStreamNonBlocking)) != cudaSuccess) {
+            release();
             return cuda_fail(e, "cudaStreamCreate(pipeline)");
+        }
         dc.ev_h2d = new std::vector<cudaEvent_t>();
         dc.ev_kernel_g = new std::vector<cudaEvent_t>();
         dc.ev_kernel_d = new std::vector<cudaEvent_t>();
         dc.ev_d2h = new std::vector<cudaEvent_t>();
         dc.pipeline_mu = new std::mutex();
-        if (!baselines.empty())
-            cudaMemcpy(dc.baselines, baselines.data(), baselines.size() * 4, cudaMemcpyHostToDevice);
-        e = cudaMemcpy(dc.frequencies, frequencies.data(), frequencies.size() * 8, cudaMemcpyHostToDevice);
-        if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy(plan)");
         auto res = device.emplace(dev, dc);
         *out = &res.first->second;
         return IDG_OK;
@@ -537,16 +545,18 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
     try {
         idg_status st = validate_call(plan, h_vis, d_uvw, d_aterms, d_taper, d_grid);
         if (st != IDG_OK) return st;
+        const size_t bl_bytes = size_t(plan->nr_timesteps) * plan->nr_channels * 32;
+        if (plan->items.empty()) {  // nothing to predict: every visibility is dropped -> 0 (no GPU work)
+            const size_t bytes = size_t(plan->nr_baselines) * bl_bytes;
+            if (bytes > 0 && !h_vis) return fail(IDG_ERR_INVALID_ARG, "h_vis is NULL");
+            if (bytes > 0) std::memset(h_vis, 0, bytes);
+            return IDG_OK;
+        }
         const size_t need = size_t(2) * kStagingBuffers * plan->group_bytes;
-        if (!plan->groups.empty() && (!d_workspace || workspace_bytes < need))
+        if (!d_workspace || workspace_bytes < need)
             return fail(IDG_ERR_WORKSPACE_TOO_SMALL, "host-streamed degridding needs idg_host_workspace_size() = " +
                                                          std::to_string(need) + " bytes");
         const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-        const size_t bl_bytes = size_t(plan->nr_timesteps) * plan->nr_channels * 32;
-        if (plan->items.empty()) {  // nothing to predict: every visibility is dropped -> 0
-            std::memset(h_vis, 0, size_t(plan->nr_baselines) * bl_bytes);
-            return IDG_OK;
-        }
         const DeviceCopy *dc = nullptr;
         if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
         std::lock_guard<std::mutex> lock(*dc->pipeline_mu);

@@ -514,7 +514,7 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 const Variant kTcGridder[] = {
     TGB(24, 12, 3, 2, 128), TG(24, 12, 3, 2), TG(24, 6, 6, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
     TG(24, 6, 6, 3), TG(24, 9, 4, 3), TG(24, 4, 9, 4),
-    TGR(32, 8, 8, 2), TGR(32, 16, 4, 2), TGR(32, 16, 4, 1),
+    TGR(32, 16, 4, 2), TGR(32, 8, 8, 2), TGR(32, 16, 4, 1),
     TG(32, 16, 4, 2), TG(32, 8, 8, 2), TG(32, 16, 4, 1), TG(32, 4, 16, 3), TG(32, 8, 8, 3),
     TG(16, 4, 4, 4), TG(16, 8, 2, 3), TG(16, 16, 1, 2),
     TGR(24, 12, 3, 2), TGR(24, 9, 4, 3), TGR(24, 6, 6, 2), TGR(24, 4, 9, 4), TGR(24, 12, 3, 1),

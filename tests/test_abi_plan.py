@@ -103,3 +103,19 @@ def test_empty_plan():
     obs0 = obs.subset(nr_baselines=0)
     plan = idg.Plan.from_observation(obs0)
     assert plan.nr_subgrids == 0 and plan.stats()["nr_pairs"] == 0
+
+
+def test_calls_on_a_plan_without_items_need_no_gpu():
+    """A plan whose visibilities are all dropped launches nothing: degridding defines them as 0 (R-12,
+    R-13) on the host path too, and a NULL host buffer is an argument error, not a crash."""
+    obs = idgsynth.make_observation("small_dde")
+    plan = idg.Plan.from_observation(dataclasses.replace(obs, image_size=1.4))  # every subgrid falls off
+    assert plan.nr_subgrids == 0 and plan.stats()["nr_vis_dropped"] == obs.nr_baselines * obs.nr_timesteps * obs.nr_channels
+    lib = idg.lib()
+    h = plan._h
+    assert lib.idg_degrid_host(h, None, None, None, None, None, None, 0, None) == 1   # IDG_ERR_INVALID_ARG
+    vis = np.full((obs.nr_baselines, obs.nr_timesteps, obs.nr_channels, 4), 1 + 1j, dtype=np.complex64)
+    assert lib.idg_degrid_host(h, None, None, None, None, vis.ctypes.data, None, 0, None) == 0
+    assert not vis.any()
+    assert lib.idg_grid_host(h, None, None, None, None, None, None, 0, None) == 0      # nothing to add
+    assert lib.idg_grid(h, None, None, None, None, None, None, 0, None) == 0
