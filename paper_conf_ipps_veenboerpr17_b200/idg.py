@@ -201,6 +201,16 @@ def _stream(stream):
     return ctypes.c_void_p(s.cuda_stream)
 
 
+def _one_device(*tensors):
+    """The single CUDA device of the call's device tensors (made current for the call: the plan's device
+    copy and the default stream are per device)."""
+    import torch
+    devs = {t.device for t in tensors if isinstance(t, torch.Tensor) and t.is_cuda}
+    if len(devs) != 1:
+        raise ValueError(f"all device tensors of a call must be on one CUDA device, got {sorted(map(str, devs))}")
+    return torch.cuda.device(devs.pop())
+
+
 def _shapes(plan: Plan):
     import torch
     n = plan.subgrid_size
@@ -217,7 +227,8 @@ def grid(plan: Plan, vis, uvw, aterms, taper, grid_out, stream=None):
     sh = _shapes(plan)
     args = [_dev(vis, *sh["vis"], "vis"), _dev(uvw, *sh["uvw"], "uvw"), _dev(aterms, *sh["aterms"], "aterms"),
             _dev(taper, *sh["taper"], "taper"), _dev(grid_out, *sh["grid"], "grid")]
-    _check(lib().idg_grid(plan.handle, *args, None, 0, _stream(stream)), "idg_grid")
+    with _one_device(vis, uvw, aterms, taper, grid_out):
+        _check(lib().idg_grid(plan.handle, *args, None, 0, _stream(stream)), "idg_grid")
     return grid_out
 
 
@@ -227,7 +238,8 @@ def degrid(plan: Plan, grid_in, uvw, aterms, taper, vis_out, stream=None):
     args = [_dev(grid_in, *sh["grid"], "grid"), _dev(uvw, *sh["uvw"], "uvw"),
             _dev(aterms, *sh["aterms"], "aterms"), _dev(taper, *sh["taper"], "taper"),
             _dev(vis_out, *sh["vis"], "vis")]
-    _check(lib().idg_degrid(plan.handle, *args, None, 0, _stream(stream)), "idg_degrid")
+    with _one_device(grid_in, uvw, aterms, taper, vis_out):
+        _check(lib().idg_degrid(plan.handle, *args, None, 0, _stream(stream)), "idg_degrid")
     return vis_out
 
 
@@ -251,14 +263,22 @@ def workspace(plan: Plan, device=None, full: bool = False):
     return torch.empty(max(1, n), dtype=torch.uint8, device=device or "cuda")
 
 
+def _workspace_ok(ws):
+    import torch
+    if not isinstance(ws, torch.Tensor) or not ws.is_cuda or ws.dtype != torch.uint8 or not ws.is_contiguous():
+        raise TypeError("ws must be a contiguous uint8 CUDA tensor (see workspace())")
+
+
 def grid_host(plan: Plan, vis_host, uvw, aterms, taper, grid_out, ws, stream=None):
     """idg_grid_host: visibilities in (pinned) host memory, streamed through `ws`."""
     sh = _shapes(plan)
     args = [_host(vis_host, *sh["vis"], "vis_host"), _dev(uvw, *sh["uvw"], "uvw"),
             _dev(aterms, *sh["aterms"], "aterms"), _dev(taper, *sh["taper"], "taper"),
             _dev(grid_out, *sh["grid"], "grid")]
-    _check(lib().idg_grid_host(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)),
-           "idg_grid_host")
+    _workspace_ok(ws)
+    with _one_device(uvw, aterms, taper, grid_out, ws):
+        _check(lib().idg_grid_host(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(),
+                                   _stream(stream)), "idg_grid_host")
     return grid_out
 
 
@@ -268,8 +288,10 @@ def degrid_host(plan: Plan, grid_in, uvw, aterms, taper, vis_host_out, ws, strea
     args = [_dev(grid_in, *sh["grid"], "grid"), _dev(uvw, *sh["uvw"], "uvw"),
             _dev(aterms, *sh["aterms"], "aterms"), _dev(taper, *sh["taper"], "taper"),
             _host(vis_host_out, *sh["vis"], "vis_host_out")]
-    _check(lib().idg_degrid_host(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(),
-                                 _stream(stream)), "idg_degrid_host")
+    _workspace_ok(ws)
+    with _one_device(grid_in, uvw, aterms, taper, ws):
+        _check(lib().idg_degrid_host(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(),
+                                     _stream(stream)), "idg_degrid_host")
     return vis_host_out
 
 
