@@ -7,7 +7,10 @@ They do not re-run the greedy algorithm; they check what any correct plan must s
   * placement: the subgrid centre cell is within half a cell of the footprint centre (R-11);
   * T~ <= T~max (P:139); no item straddles an A-term slot and aterm_index is the slot of t0 (R-15);
   * greedy maximality: an item that could have been extended (same slot, below T~max, not at T)
-    would NOT fit with one more timestep ("as many time steps as possible").
+    would NOT fit with one more timestep ("as many time steps as possible", P:137);
+  * drops are forced: every visibility left out belongs to a (baseline, timestep, channel block) that
+    cannot form an item on its own — its footprint + K exceeds N~ (R-13) or its subgrid falls off the
+    grid (R-12) — so a plan cannot pass by dropping data it could have gridded.
 Shared by the oracle-plan tests (CPU) and the library-plan tests.
 """
 import numpy as np
@@ -68,4 +71,16 @@ def check_plan(obs, items, nr_dropped, check_maximal=True):
                 assert not fits, f"item {it} is not maximal"
     assert cover.max(initial=0) <= 1, "visibility in two items"
     assert int((cover == 0).sum()) == nr_dropped, (int((cover == 0).sum()), nr_dropped)
+    cb = obs.max_channels_per_subgrid or C
+    for c0 in range(0, C, cb):
+        c1 = min(C, c0 + cb)
+        blk = cover[:, :, c0:c1]
+        assert np.all((blk == 0).all(axis=2) | (blk == 1).all(axis=2)), "channel block split across items"
+        for b, t in zip(*np.nonzero((blk == 0).all(axis=2))):
+            uu, vv = u[b, t, c0:c1], v[b, t, c0:c1]
+            too_wide = (uu.max() - uu.min()) + K > n or (vv.max() - vv.min()) + K > n
+            x = np.floor((uu.max() + uu.min()) / 2 + N / 2 + 0.5) - n / 2
+            y = np.floor((vv.max() + vv.min()) / 2 + N / 2 + 0.5) - n / 2
+            off_grid = not (0 <= x and x + n <= N and 0 <= y and y + n <= N)
+            assert too_wide or off_grid, f"baseline {b} timestep {t} channels [{c0},{c1}) dropped but fits"
     return cover

@@ -56,3 +56,21 @@ def test_plan_w_planes(nz):
     items, dropped = oracle.plan(obs)
     check_plan(obs, items, dropped)
     assert len(set(items["z"].tolist())) >= 2
+
+
+def test_plan_checks_reject_unforced_drops():
+    """Mutation test of the checker: dropping one gridable item (and counting its visibilities as
+    dropped) must be caught, as must shortening an item (breaks maximality)."""
+    obs = idgsynth.make_observation("small_dde")
+    items, dropped = oracle.plan(obs)
+    victim = items[len(items) // 2]
+    nvis = int(victim["nr_timesteps"]) * int(victim["channel_end"] - victim["channel_begin"])
+    fewer = np.delete(items, len(items) // 2)
+    with pytest.raises(AssertionError, match="dropped but fits"):
+        check_plan(obs, fewer, dropped + nvis)
+    shorter = items.copy()
+    k = int(np.argmax(items["nr_timesteps"]))
+    shorter[k]["nr_timesteps"] -= 1
+    nc = int(items[k]["channel_end"] - items[k]["channel_begin"])
+    with pytest.raises(AssertionError):
+        check_plan(obs, shorter, dropped + nc)
