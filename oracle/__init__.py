@@ -51,9 +51,11 @@ _lib = None
 
 
 def lib():
+    """The compiled oracle.  IDG_ORACLE_LIB (test infrastructure: tests/test_oracle_mutants.py) loads a
+    mutated build of idg_oracle.c instead, to show that the pins reject it."""
     global _lib
     if _lib is None:
-        _lib = ctypes.CDLL(build())
+        _lib = ctypes.CDLL(os.environ.get("IDG_ORACLE_LIB") or build())
         P = ctypes.c_void_p
         i32, i64 = ctypes.c_int32, ctypes.c_int64
         _lib.oracle_plan.restype = i64
