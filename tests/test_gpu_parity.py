@@ -242,3 +242,27 @@ def test_full_size_configs_sampled(name):
     torch.cuda.synchronize()
     lhs, rhs = _inner_t(DG, V), _inner_t(G, gV)
     assert abs(lhs - rhs) / abs(lhs) < 1e-4, (lhs, rhs)
+
+
+def test_tolerance_is_discriminating():
+    """The 1e-4 bar is tight enough to see small systematic errors: the kernels' own error is far below
+    it, while a 2e-5 relative uvw scale error, a one-timestep shift of the visibilities or two swapped
+    polarisations -- fed to the same GPU path -- exceed it."""
+    obs = idgsynth.make_observation("lofar_dde", T=512, nr_stations=5)
+    vis, aterms, taper = _inputs(obs)
+    items, _ = oracle.plan(obs)
+    ref = oracle.grid(obs, items, vis, aterms, taper)
+    plan = idg.Plan.from_observation(obs)
+    good = rel_rms(gpu_grid(obs, vis, aterms, taper, plan).cpu().numpy(), ref)
+    assert good < TOL / 5, good
+
+    def err_with(uvw=None, v=None):
+        g = torch.zeros(oracle.grid_shape(obs), dtype=torch.complex64, device="cuda")
+        idg.grid(plan, _dev(vis if v is None else v), _dev(obs.uvw if uvw is None else uvw), _dev(aterms),
+                 _dev(taper), g)
+        torch.cuda.synchronize()
+        return rel_rms(g.cpu().numpy(), ref)
+
+    assert err_with(uvw=(obs.uvw * (1 + 2e-5)).astype(np.float32)) > TOL
+    assert err_with(v=np.roll(vis, 1, axis=1)) > TOL
+    assert err_with(v=vis[..., [0, 2, 1, 3]]) > TOL
