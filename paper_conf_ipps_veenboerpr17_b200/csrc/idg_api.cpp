@@ -361,11 +361,13 @@ idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, i
         }
         plan->channel_gcd = g == 0 ? 1 : g;
         // uniform channel spacing (enables the phasor recurrence over channels in the gridder)
+        // (every nu_c within 1e-12 nu_0 of nu_0 + c d: the kernels that rotate phasors across channels
+        // then see phase errors below 2 pi |u| 1e-12 nu_0 C / c * L/2 ~ 1e-6 rad at the configs)
         if (nr_channels >= 2) {
-            const double d0 = frequencies[1] - frequencies[0];
+            const double d0 = (frequencies[nr_channels - 1] - frequencies[0]) / double(nr_channels - 1);
             bool uni = d0 != 0.0;
-            for (int32_t c = 1; c + 1 < nr_channels && uni; ++c)
-                uni = std::fabs((frequencies[c + 1] - frequencies[c]) - d0) <= 1e-9 * std::fabs(frequencies[0]);
+            for (int32_t c = 1; c < nr_channels && uni; ++c)
+                uni = std::fabs(frequencies[c] - (frequencies[0] + double(c) * d0)) <= 1e-12 * std::fabs(frequencies[0]);
             plan->channels_uniform = uni ? 1 : 0;
             plan->channel_step = float(d0 / idg::kSpeedOfLight);
         }

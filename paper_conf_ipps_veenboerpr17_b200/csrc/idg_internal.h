@@ -49,7 +49,7 @@ struct KernelArgs {
     int32_t max_channels_in_item;
     int32_t max_timesteps_in_item;
     int32_t channel_gcd;         // gcd of all items' channel counts
-    int32_t channels_uniform;    // 1 if nu_{c+1} - nu_c is the same for all c (to 1e-9 relative)
+    int32_t channels_uniform;    // 1 if nu_c = nu_0 + c d for all c (to 1e-12 nu_0)
     float channel_step;          // (nu_{c+1} - nu_c) / c  [1/m], valid when channels_uniform
 };
 
@@ -62,6 +62,7 @@ struct Variant {
     int needs_uniform; // 1: requires uniformly spaced channels (phasor recurrence over channels)
     const char *name;
     Launcher fn;
+    int max_channels = 0;  // > 0: every item has at most this many channels (unrolled channel groups)
 };
 // Tensor-core variants (idg_kernels_tc.cu); the first eligible one is the default.
 const Variant *tc_gridder_variants(int *n);     // split-f16 mma (idg_kernels_tc.cu)

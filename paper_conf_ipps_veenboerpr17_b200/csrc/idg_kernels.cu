@@ -319,6 +319,7 @@ const Variant kDegridderVariants[] = {DV_ALL(24), DV_ALL(32), DV_ALL(16)};
 bool eligible(const Variant &var, const KernelArgs &a) {
     if (var.ns != a.subgrid_size) return false;
     if (var.needs_uniform && !a.channels_uniform) return false;
+    if (var.max_channels > 0 && a.max_channels_in_item > var.max_channels) return false;
     return var.v == 0 || a.channel_gcd % var.v == 0;
 }
 

@@ -85,6 +85,16 @@ __device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1
         : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
 }
 
+// D = A B (fresh accumulator: C = 0).
+__device__ __forceinline__ void mma16816_zero(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
+                                              uint32_t b0, uint32_t b1) {
+    const float z = 0.0f;
+    asm("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%10,%10,%10,%10};"
+        : "=f"(d[0]), "=f"(d[1]), "=f"(d[2]), "=f"(d[3])
+        : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1), "f"(z));
+}
+
 // The three split products of one tile: D += Ahi Bhi + Ahi Blo + Alo Bhi.
 __device__ __forceinline__ void mma3(float (&d)[4], const uint32_t (&ah)[4], const uint32_t (&al)[4],
                                      const uint4 &b) {
@@ -327,6 +337,199 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
 }
 
 // ------------------------------------------------------------------------------------------------
+// Tensor-core gridder with accumulator rotation across channel groups (uniformly spaced channels).
+//
+// The phase is linear in frequency (R-2: phi = B_t + (nu_c/c - f_ref) Q_t), so with channels
+// c = 8j + s (group j = 0..J-1, slot s = 0..7, J = C~/8) and spacing dnu,
+//     Phi(t, 8j + s) = Phi(t, s) E_t^j,    E_t = exp(i 8 dnu/c Q_t)    (per pixel and timestep)
+// and the per-timestep contribution to a pixel factorises:
+//     sum_c Phi(t,c) V(t,c) = sum_j E_t^j D_j,   D_j = sum_s Phi(t,s) V(t, 8j+s).
+// Every D_j is an mma of the SAME A fragment (the slot-s phasors of group 0) with group j's B fragment,
+// so the sincos + split work per (pixel, timestep) is that of 8 visibilities plus one sincos for E_t,
+// instead of C~.  D_j is formed fresh per timestep (split-f16, three products) and rotated into the
+// fp32 accumulator with E_t^j (E_t^j by recurrence).  Exact in exact arithmetic; the rounding is that of
+// one extra complex product per (pixel, timestep, group).  Batches hold whole timesteps.
+// ------------------------------------------------------------------------------------------------
+inline size_t gridder_rot_smem_bytes(int NS, int kbb_ = kTcBatchKB) {
+    const size_t kbb = kbb_;
+    const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + (kbb + 1) * 32 /*coef*/;
+    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2);
+    return std::max(main, epi) + 16;
+}
+
+template <int NS, int WARPS, int MT, int MINB, int KPT, int KBB_ = kTcBatchKB>
+__global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot_kernel(const KernelArgs a) {
+    constexpr int NT = WARPS * 32;
+    constexpr int NPIX = NS * NS;
+    static_assert(WARPS * MT * 16 == NPIX, "warps x m-tiles x 16 must cover the subgrid");
+    static_assert(KPT >= 1 && KPT <= KBB_, "channel groups per timestep");
+    constexpr int h = NS / 2;
+    constexpr int KBB = KBB_;
+    constexpr int VB = KBB * 8;
+    extern __shared__ __align__(16) unsigned char smem[];
+    float4 *raw_s = reinterpret_cast<float4 *>(smem);                // [VB][2]
+    uint4 *frag_s = reinterpret_cast<uint4 *>(raw_s + 2 * VB);       // [KBB][32]
+    float4 *coef_s = reinterpret_cast<float4 *>(frag_s + KBB * 32);  // [KBB+1][2]
+    __shared__ float red_s[WARPS];
+    __shared__ float2 tw[NS];
+
+    const int item = a.order[blockIdx.x];
+    const ItemSetup s = dev::item_setup(a, item, NS);
+    const idg_metadata &md = s.md;
+    const int nc = s.nc;
+    const int kpt = nc >> 3;                     // channel groups (k-blocks) per timestep, <= KPT
+    const int tpb = KBB / kpt;                   // whole timesteps per batch
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
+
+    // slots q and q+4 of group 0 (channel offsets from the reference frequency) and the group step
+    const f2p dq = dup(float(a.frequencies[md.channel_begin + q] / kSpeedOfLight - s.f_ref));
+    const f2p dq4 = dup(float(a.frequencies[md.channel_begin + q + 4] / kSpeedOfLight - s.f_ref));
+    const f2p est = dup(8.0f * a.channel_step);
+
+    f2p pl[MT], pm[MT], pn[MT];
+    float acc[MT][4];
+#pragma unroll
+    for (int i = 0; i < MT; ++i) {
+        float l2[2], m2[2], n2[2];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            const int pix = (warp * MT + i) * 16 + g + 8 * r;
+            const int x = pix % NS, y = pix / NS;
+            l2[r] = float(x - h) * a.cell_l;
+            m2[r] = float(y - h) * a.cell_l;
+            n2[r] = dev::w_term_n(l2[r], m2[r]);
+        }
+        pl[i] = pk(l2[0], l2[1]);
+        pm[i] = pk(m2[0], m2[1]);
+        pn[i] = pk(n2[0], n2[1]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
+    }
+    float cur_scale = 0.0f;
+
+    const int64_t row = int64_t(a.nr_channels) * 4;  // float2 per timestep
+    const float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
+                         int64_t(md.channel_begin) * 4;
+
+    for (int t0 = 0; t0 < md.nr_timesteps; t0 += tpb) {
+        const int t1 = min(t0 + tpb, md.nr_timesteps);
+        const int nkb = (t1 - t0) * kpt;
+        const int nvb = nkb * 8;
+        __syncthreads();  // previous batch fully consumed
+        // (1) raw visibilities of timesteps [t0, t1): index j = (t - t0) nc + c
+        for (int i = threadIdx.x; i < 2 * nvb; i += NT) {
+            const int j = i >> 1;
+            const int t = j / nc, c = j - t * nc;
+            raw_s[i] = dev::ld_stream(reinterpret_cast<const float4 *>(vis0 + int64_t(t0 + t) * row + c * 4) + (i & 1));
+        }
+        // (2) per-timestep phase coefficients (fp64 -> fp32)
+        for (int t = t0 + int(threadIdx.x); t < t1; t += NT) {
+            float4 cB, cQ;
+            dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
+            coef_s[2 * (t - t0)] = cB;
+            coef_s[2 * (t - t0) + 1] = cQ;
+        }
+        __syncthreads();
+        // (3) f16 range: power-of-two scale from the batch maximum; never increase the running scale
+        float mx = 0.0f;
+        for (int i = threadIdx.x; i < 2 * nvb; i += NT) mx = abs_max4(raw_s[i], mx).x;
+        const float bscale = pow2_scale(block_max<WARPS>(mx, red_s));
+        if (cur_scale == 0.0f) {
+            cur_scale = bscale;
+        } else if (bscale < cur_scale) {
+            const float f = bscale / cur_scale;  // exact power of two
+#pragma unroll
+            for (int i = 0; i < MT; ++i)
+#pragma unroll
+                for (int j = 0; j < 4; ++j) acc[i][j] *= f;
+            cur_scale = bscale;
+        }
+        // (4) B fragments of every (timestep, group): column g = 2 pol + im, k-slots q and q+4
+        for (int i = threadIdx.x; i < nkb * 32; i += NT) {
+            const int kbl = i >> 5, ln = i & 31, gg = ln >> 2, qq = ln & 3;
+            const int pol = gg >> 1, im = gg & 1;
+            uint32_t hi[2], lo[2];
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const float4 v4 = raw_s[2 * (kbl * 8 + qq + 4 * r) + (pol >> 1)];
+                const float vr = ((pol & 1) ? v4.z : v4.x) * cur_scale;
+                const float vi = ((pol & 1) ? v4.w : v4.y) * cur_scale;
+                split2(im ? vi : vr, im ? vr : -vi, hi[r], lo[r]);
+            }
+            frag_s[i] = make_uint4(hi[0], hi[1], lo[0], lo[1]);
+        }
+        __syncthreads();
+        // (5) per timestep: group-0 phasors of every tile, E_t, and one fresh D_j per group
+#pragma unroll 1
+        for (int t = t0; t < t1; ++t) {
+            const float4 cB = coef_s[2 * (t - t0)], cQ = coef_s[2 * (t - t0) + 1];
+            const uint4 *fr = frag_s + (t - t0) * kpt * 32 + lane;
+#pragma unroll
+            for (int i = 0; i < MT; ++i) {
+                const f2p Bv = fma2(dup(cB.x), pl[i], fma2(dup(cB.y), pm[i], mul2(dup(cB.z), pn[i])));
+                const f2p Qv = fma2(dup(cQ.x), pl[i], fma2(dup(cQ.y), pm[i], mul2(dup(cQ.z), pn[i])));
+                const float2 ph0 = unpk(fma2(dq, Qv, Bv));    // (row g, row g+8) at slot q
+                const float2 ph1 = unpk(fma2(dq4, Qv, Bv));   // (row g, row g+8) at slot q+4
+                float sn[4], cs[4];
+                __sincosf(ph0.x, &sn[0], &cs[0]);
+                __sincosf(ph0.y, &sn[1], &cs[1]);
+                __sincosf(ph1.x, &sn[2], &cs[2]);
+                __sincosf(ph1.y, &sn[3], &cs[3]);
+                uint32_t ah[4], al[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[j], al[j]);
+                float er0 = 1.0f, ei0 = 0.0f, er1 = 1.0f, ei1 = 0.0f;  // E_t of rows g, g+8
+                if (KPT > 1 && kpt > 1) {
+                    const float2 e = unpk(mul2(est, Qv));
+                    __sincosf(e.x, &ei0, &er0);
+                    __sincosf(e.y, &ei1, &er1);
+                }
+                float pr0 = 1.0f, pi0 = 0.0f, pr1 = 1.0f, pi1 = 0.0f;  // E_t^j
+#pragma unroll
+                for (int j = 0; j < KPT; ++j) {
+                    if (j > 0 && j >= kpt) break;
+                    const uint4 bf = fr[j * 32];
+                    float d[4];
+                    mma16816_zero(d, ah[0], ah[1], ah[2], ah[3], bf.x, bf.y);
+                    mma16816(d, ah[0], ah[1], ah[2], ah[3], bf.z, bf.w);
+                    mma16816(d, al[0], al[1], al[2], al[3], bf.x, bf.y);
+                    if (j == 0) {
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) acc[i][k] += d[k];
+                    } else {
+                        if (j == 1) {
+                            pr0 = er0; pi0 = ei0; pr1 = er1; pi1 = ei1;
+                        } else {
+                            const float a0 = fmaf(pr0, er0, -pi0 * ei0), b0 = fmaf(pr0, ei0, pi0 * er0);
+                            const float a1 = fmaf(pr1, er1, -pi1 * ei1), b1 = fmaf(pr1, ei1, pi1 * er1);
+                            pr0 = a0; pi0 = b0; pr1 = a1; pi1 = b1;
+                        }
+                        acc[i][0] = fmaf(pr0, d[0], fmaf(-pi0, d[1], acc[i][0]));
+                        acc[i][1] = fmaf(pr0, d[1], fmaf(pi0, d[0], acc[i][1]));
+                        acc[i][2] = fmaf(pr1, d[2], fmaf(-pi1, d[3], acc[i][2]));
+                        acc[i][3] = fmaf(pr1, d[3], fmaf(pi1, d[2], acc[i][3]));
+                    }
+                }
+            }
+        }
+    }
+
+    // ---- epilogue: D fragments -> sub_s[pol][pixel], then a3 + a4 + a5 ---------------------------
+    __syncthreads();
+    float2 *sub_s = reinterpret_cast<float2 *>(smem);
+    float2 *tmp_s = sub_s + 4 * NPIX;
+    const float inv = cur_scale > 0.0f ? 1.0f / cur_scale : 1.0f;
+#pragma unroll
+    for (int i = 0; i < MT; ++i) {
+        const int p0 = (warp * MT + i) * 16 + g;
+        sub_s[q * NPIX + p0] = make_float2(acc[i][0] * inv, acc[i][1] * inv);
+        sub_s[q * NPIX + p0 + 8] = make_float2(acc[i][2] * inv, acc[i][3] * inv);
+    }
+    __syncthreads();
+    dev::gridder_epilogue<NS>(a, s, sub_s, tmp_s, tw);
+}
+
+// ------------------------------------------------------------------------------------------------
 // Tensor-core degridder.  One CTA per work item.  Prologue (a6-a8) leaves the corrected subgrid as
 // B fragments (k-block = 8 pixels) + per-pixel {l, m, n}; m-tile = 16 consecutive visibilities of
 // the item (flattened (t, c) order); each warp takes MT tiles at a time over all k-blocks.
@@ -334,7 +537,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
 inline size_t degridder_tc_smem_bytes(int NS, int max_timesteps, int max_channels) {
     const size_t npix = size_t(NS) * NS;
     return npix * 64 /*sub+tmp | frag*/ + npix * 4 * 8 / 2 /*lmn slot pairs: 32 B per 2 pixels*/ +
-           size_t(max_timesteps) * 16 /*uvw of the item's timesteps*/ + size_t(max_channels) * 8 /*nu/c*/ + 16;
+           size_t(max_timesteps) * 32 /*B_t, Q_t of the item's timesteps*/ + size_t(max_channels) * 4 /*df*/ + 16;
 }
 
 template <int NS, int WARPS, int MT, int MINB>
@@ -350,8 +553,8 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     float2 *tmp_s = sub_s + 4 * NPIX;                                     // [4][NS][NS]
     uint4 *frag_s = reinterpret_cast<uint4 *>(smem);                      // [NKB][32] (after prologue)
     float4 *lmn_s = reinterpret_cast<float4 *>(smem + size_t(NPIX) * 64); // [NKB][4][2] slot pairs
-    float4 *uvw_s = lmn_s + NKB * 8;                                      // [T~]: u, v, w of the item
-    double *fq_s = reinterpret_cast<double *>(uvw_s + a.max_timesteps_in_item);  // [C~]: nu / c
+    float4 *bq_s = lmn_s + NKB * 8;                                       // [T~][2]: B_t, Q_t of the item
+    float *df_s = reinterpret_cast<float *>(bq_s + 2 * a.max_timesteps_in_item);  // [C~]: nu/c - f_ref
     __shared__ float red_s[WARPS];
     __shared__ float2 tw[NS];
 
@@ -361,14 +564,18 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     const int nc = s.nc;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
 
-    // the item's uvw and nu/c, read by every tile's phase coefficients (staged once: no dependent
-    // global loads in front of each tile's k-block loop)
+    // per-timestep phase coefficients B_t = 2 pi (uvw_t f_ref - uvw0), Q_t = 2 pi uvw_t (fp64 -> fp32,
+    // once per item) and channel offsets df_c = nu_c/c - f_ref: a visibility's coefficients are then
+    // B_t + df_c Q_t (fp32 FMAs, as in the gridder), with no fp64 work in front of each tile
     for (int t = threadIdx.x; t < md.nr_timesteps; t += NT) {
-        const float *p = a.uvw + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset + t) * 3;
-        uvw_s[t] = make_float4(p[0], p[1], p[2], 0.0f);
+        float4 cB, cQ;
+        dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
+        bq_s[2 * t] = cB;
+        bq_s[2 * t + 1] = cQ;
     }
-    for (int c = threadIdx.x; c < nc; c += NT) fq_s[c] = a.frequencies[md.channel_begin + c] / kSpeedOfLight;
-    dev::degridder_split_columns<NS>(a, s, sub_s, tmp_s, tw);  // (its barriers publish uvw_s / fq_s)
+    for (int c = threadIdx.x; c < nc; c += NT)
+        df_s[c] = float(a.frequencies[md.channel_begin + c] / kSpeedOfLight - s.f_ref);
+    dev::degridder_split_columns<NS>(a, s, sub_s, tmp_s, tw);  // (its barriers publish bq_s / df_s)
     float2 rr[PPT][4];
     float mx = 0.0f;
 #pragma unroll
@@ -414,6 +621,11 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 
     const int nvis = md.nr_timesteps * nc;
     const int ntiles = (nvis + 15) >> 4;
+    // t = v / nc without an integer division: (v + 1/2) / nc is at least 1/(2 nc) away from an integer,
+    // and the fp32 quotient's error (v / nc) 2^-23 is smaller for v < 2^22 (else: integer division)
+    const float rnc = 1.0f / float(nc);
+    const bool fdiv = nvis < (1 << 22);
+    auto tstep = [&](int v) { return fdiv ? __float2int_rz((float(v) + 0.5f) * rnc) : v / nc; };
     const int64_t row = int64_t(a.nr_channels) * 4;
     float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
                    int64_t(md.channel_begin) * 4;
@@ -427,12 +639,12 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
                 const int v = (tile0 + i) * 16 + g + 8 * r;
                 float fu = 0.0f, fv = 0.0f, fw = 0.0f;
                 if (v < nvis) {
-                    const int t = v / nc, c = v - t * nc;
-                    const float4 p = uvw_s[t];
-                    const double f = fq_s[c];
-                    fu = float(dev::kTwoPi * (double(p.x) * f - s.u0));
-                    fv = float(dev::kTwoPi * (double(p.y) * f - s.v0));
-                    fw = float(dev::kTwoPi * (double(p.z) * f - s.w0));
+                    const int t = tstep(v), c = v - t * nc;
+                    const float4 cB = bq_s[2 * t], cQ = bq_s[2 * t + 1];
+                    const float df = df_s[c];
+                    fu = fmaf(df, cQ.x, cB.x);
+                    fv = fmaf(df, cQ.y, cB.y);
+                    fw = fmaf(df, cQ.z, cB.z);
                 }
                 cu[i][r] = dup(fu);
                 cv[i][r] = dup(fv);
@@ -473,7 +685,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
             for (int r = 0; r < 2; ++r) {
                 const int v = (tile0 + i) * 16 + g + 8 * r;
                 if (v < nvis) {
-                    const int t = v / nc, c = v - t * nc;
+                    const int t = tstep(v), c = v - t * nc;
                     vis0[int64_t(t) * row + c * 4 + q] = make_float2(acc[i][2 * r] * inv, acc[i][2 * r + 1] * inv);
                 }
             }
@@ -488,6 +700,16 @@ cudaError_t launch_gridder_tc(const KernelArgs &a, cudaStream_t st) {
     if (err != cudaSuccess) return err;
     LaunchScope scope("gridder", st);
     gridder_tc_kernel<NS, WARPS, MT, MINB, REC, KBB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+template <int NS, int WARPS, int MT, int MINB, int KPT, int KBB = kTcBatchKB>
+cudaError_t launch_gridder_rot(const KernelArgs &a, cudaStream_t st) {
+    const size_t smem = gridder_rot_smem_bytes(NS, KBB);
+    cudaError_t err = dev::prepare(gridder_rot_kernel<NS, WARPS, MT, MINB, KPT, KBB>, smem);
+    if (err != cudaSuccess) return err;
+    LaunchScope scope("gridder", st);
+    gridder_rot_kernel<NS, WARPS, MT, MINB, KPT, KBB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -511,7 +733,13 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 // channel-recurrence kernel run within 2% of each other (the kernels are latency-bound below the
 // XU limit), so the direct kernel (no recurrence error) is the default for N~ = 24; for N~ = 32 the
 // recurrence variant is 1% faster.
+#define TGROT(NS, W, MT, MB, KPT) \
+    {NS, 8, kTensor, 1, "gridder_rot<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ">", \
+     launch_gridder_rot<NS, W, MT, MB, KPT, 128>, 8 * KPT}
 const Variant kTcGridder[] = {
+    TGROT(24, 12, 3, 2, 4), TGROT(24, 12, 3, 2, 2), TGROT(24, 12, 3, 1, 2), TGROT(24, 12, 3, 1, 4),
+    TGROT(32, 16, 4, 1, 4), TGROT(32, 16, 4, 1, 2), TGROT(32, 8, 8, 1, 4), TGROT(32, 16, 4, 1, 8),
+    TGROT(16, 8, 2, 2, 2), TGROT(16, 8, 2, 2, 4), TGROT(24, 12, 3, 1, 8),
     TGB(24, 12, 3, 2, 128), TG(24, 12, 3, 2), TG(24, 6, 6, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
     TG(24, 6, 6, 3), TG(24, 9, 4, 3), TG(24, 4, 9, 4),
     TGR(32, 16, 4, 2), TGR(32, 8, 8, 2), TGR(32, 16, 4, 1),
@@ -523,6 +751,7 @@ const Variant kTcGridder[] = {
 };
 #undef TGB
 #undef TGR
+#undef TGROT
 #undef TG
 #define TD(NS, W, MT, MB) \
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>}

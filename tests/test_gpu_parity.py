@@ -74,6 +74,7 @@ KINDS = {
     "default": (None, None),                       # default tensor-core kernels (split-f16 mma)
     "tc": ("tc", "tc"),                            # direct tensor-core kernels (no channel recurrence)
     "rec": ("gridder_tcr<*", "degridder_tc<*"),    # split-f16 gridder with the channel recurrence
+    "rot": ("gridder_rot<*", "degridder_tc<*"),    # split-f16 gridder with accumulator rotation over channel groups
     "tf32": ("gridder_tf32*", "degridder_tf32*"),  # split-tf32 tensor-core kernels
     "umma": ("gridder_umma*", "degridder_tc<*"),    # tcgen05 / TMEM gridder
     "simt": ("simt", "simt"),                      # CUDA-core kernels (the paper's structure)
