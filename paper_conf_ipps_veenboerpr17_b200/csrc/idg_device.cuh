@@ -100,6 +100,41 @@ __device__ __forceinline__ void timestep_coefficients(const KernelArgs &a, const
 }
 
 
+// a3 for one pixel, in place: sub_s[pol][pix] <- sph * A_p^H S A_q (R-6).  Returns max |component|.
+template <int NS>
+__device__ __forceinline__ float gridder_aterm_pixel(const KernelArgs &a, const ItemSetup &s, float2 *sub_s, int pix) {
+    constexpr int NPIX = NS * NS;
+    const idg_metadata &md = s.md;
+    const float2 *Ap_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st1) * NPIX) * 4;
+    const float2 *Aq_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st2) * NPIX) * 4;
+    const float4 *ap4 = reinterpret_cast<const float4 *>(Ap_base + int64_t(pix) * 4);
+    const float4 *aq4 = reinterpret_cast<const float4 *>(Aq_base + int64_t(pix) * 4);
+    const float4 ap01 = ap4[0], ap23 = ap4[1], aq01 = aq4[0], aq23 = aq4[1];
+    const float2 p0 = make_float2(ap01.x, ap01.y), p1 = make_float2(ap01.z, ap01.w);
+    const float2 p2 = make_float2(ap23.x, ap23.y), p3 = make_float2(ap23.z, ap23.w);
+    const float2 q0 = make_float2(aq01.x, aq01.y), q1 = make_float2(aq01.z, aq01.w);
+    const float2 q2 = make_float2(aq23.x, aq23.y), q3 = make_float2(aq23.z, aq23.w);
+    const float2 s0 = sub_s[0 * NPIX + pix], s1 = sub_s[1 * NPIX + pix];
+    const float2 s2 = sub_s[2 * NPIX + pix], s3 = sub_s[3 * NPIX + pix];
+    // M = A_p^H S
+    const float2 m0 = cadd(cmulc(p0, s0), cmulc(p2, s2));
+    const float2 m1 = cadd(cmulc(p0, s1), cmulc(p2, s3));
+    const float2 m2 = cadd(cmulc(p1, s0), cmulc(p3, s2));
+    const float2 m3 = cadd(cmulc(p1, s1), cmulc(p3, s3));
+    // R = sph * M A_q
+    const float sph = a.taper[pix];
+    const float2 r0 = cscale(cadd(cmul(m0, q0), cmul(m1, q2)), sph);
+    const float2 r1 = cscale(cadd(cmul(m0, q1), cmul(m1, q3)), sph);
+    const float2 r2 = cscale(cadd(cmul(m2, q0), cmul(m3, q2)), sph);
+    const float2 r3 = cscale(cadd(cmul(m2, q1), cmul(m3, q3)), sph);
+    sub_s[0 * NPIX + pix] = r0;
+    sub_s[1 * NPIX + pix] = r1;
+    sub_s[2 * NPIX + pix] = r2;
+    sub_s[3 * NPIX + pix] = r3;
+    return fmaxf(fmaxf(fmaxf(fabsf(r0.x), fabsf(r0.y)), fmaxf(fabsf(r1.x), fabsf(r1.y))),
+                 fmaxf(fmaxf(fabsf(r2.x), fabsf(r2.y)), fmaxf(fabsf(r3.x), fabsf(r3.y))));
+}
+
 // ------------------------------------------------------------------------------------------------
 // a3 + a4 + a5 (gridder epilogue).  On entry (after a barrier) sub_s[pol][pix] holds the raw image-
 // domain sums S of the item.  Applies sph * A_p^H S A_q per pixel (R-6), the centred forward DFT
@@ -112,30 +147,7 @@ __device__ __forceinline__ void gridder_epilogue(const KernelArgs &a, const Item
     const int nt = blockDim.x;
     const idg_metadata &md = s.md;
     init_twiddles<NS>(tw, -1.0f);
-    const float2 *Ap_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st1) * NPIX) * 4;
-    const float2 *Aq_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st2) * NPIX) * 4;
-    for (int pix = threadIdx.x; pix < NPIX; pix += nt) {
-        const float4 *ap4 = reinterpret_cast<const float4 *>(Ap_base + int64_t(pix) * 4);
-        const float4 *aq4 = reinterpret_cast<const float4 *>(Aq_base + int64_t(pix) * 4);
-        const float4 ap01 = ap4[0], ap23 = ap4[1], aq01 = aq4[0], aq23 = aq4[1];
-        const float2 p0 = make_float2(ap01.x, ap01.y), p1 = make_float2(ap01.z, ap01.w);
-        const float2 p2 = make_float2(ap23.x, ap23.y), p3 = make_float2(ap23.z, ap23.w);
-        const float2 q0 = make_float2(aq01.x, aq01.y), q1 = make_float2(aq01.z, aq01.w);
-        const float2 q2 = make_float2(aq23.x, aq23.y), q3 = make_float2(aq23.z, aq23.w);
-        const float2 s0 = sub_s[0 * NPIX + pix], s1 = sub_s[1 * NPIX + pix];
-        const float2 s2 = sub_s[2 * NPIX + pix], s3 = sub_s[3 * NPIX + pix];
-        // M = A_p^H S
-        const float2 m0 = cadd(cmulc(p0, s0), cmulc(p2, s2));
-        const float2 m1 = cadd(cmulc(p0, s1), cmulc(p2, s3));
-        const float2 m2 = cadd(cmulc(p1, s0), cmulc(p3, s2));
-        const float2 m3 = cadd(cmulc(p1, s1), cmulc(p3, s3));
-        // R = sph * M A_q
-        const float sph = a.taper[pix];
-        sub_s[0 * NPIX + pix] = cscale(cadd(cmul(m0, q0), cmul(m1, q2)), sph);
-        sub_s[1 * NPIX + pix] = cscale(cadd(cmul(m0, q1), cmul(m1, q3)), sph);
-        sub_s[2 * NPIX + pix] = cscale(cadd(cmul(m2, q0), cmul(m3, q2)), sph);
-        sub_s[3 * NPIX + pix] = cscale(cadd(cmul(m2, q1), cmul(m3, q3)), sph);
-    }
+    for (int pix = threadIdx.x; pix < NPIX; pix += nt) gridder_aterm_pixel<NS>(a, s, sub_s, pix);
     __syncthreads();
     // rows: tmp[pol][y][kx] = sum_x sub[pol][y][x] exp(-2 pi i (kx-h)(x-h)/N~)
     for (int o = threadIdx.x; o < 4 * NPIX; o += nt) {
@@ -213,12 +225,15 @@ __device__ __forceinline__ void degridder_split_columns(const KernelArgs &a, con
     __syncthreads();
 }
 
+template <int NS>
+__device__ __forceinline__ void degridder_aterm_pixel(const KernelArgs &a, const ItemSetup &s, const float2 sv[4],
+                                                      int pix, float2 r[4]);
+
 // a7 (second half) + a8 for one pixel: inverse-DFT row, then sph * A_p S A_q^H (Alg. 2 lines 2-3).
 template <int NS>
 __device__ __forceinline__ void degridder_pixel(const KernelArgs &a, const ItemSetup &s, const float2 *tmp_s,
                                                 const float2 *tw, int pix, float2 r[4]) {
     constexpr int NPIX = NS * NS;
-    const idg_metadata &md = s.md;
     const int y = pix / NS, x = pix - y * NS;
     int idx0, step;
     dft_index<NS>(x, idx0, step);
@@ -239,6 +254,15 @@ __device__ __forceinline__ void degridder_pixel(const KernelArgs &a, const ItemS
         }
         sv[pol] = sum;
     }
+    degridder_aterm_pixel<NS>(a, s, sv, pix, r);
+}
+
+// a8 for one pixel: r = sph * A_p S A_q^H (Alg. 2 lines 2-3; Eq. 1: A_p B A_q^H).
+template <int NS>
+__device__ __forceinline__ void degridder_aterm_pixel(const KernelArgs &a, const ItemSetup &s, const float2 sv[4],
+                                                      int pix, float2 r[4]) {
+    constexpr int NPIX = NS * NS;
+    const idg_metadata &md = s.md;
     const float2 *Ap_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st1) * NPIX) * 4;
     const float2 *Aq_base = a.aterms + ((int64_t(md.aterm_index) * a.nr_stations + s.st2) * NPIX) * 4;
     const float4 *ap4 = reinterpret_cast<const float4 *>(Ap_base + int64_t(pix) * 4);

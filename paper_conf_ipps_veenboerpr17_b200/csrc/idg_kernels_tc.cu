@@ -129,6 +129,144 @@ __device__ __forceinline__ float4 abs_max4(float4 v, float m) {
 }
 
 // ------------------------------------------------------------------------------------------------
+// Subgrid DFT on the tensor cores (a4 / a7).  The centred 2-D DFT (R-5) is two passes of a complex
+// matrix product with the DFT matrix F[x][k] = exp(sign 2 pi i (k - N~/2)(x - N~/2) / N~):
+//     out[r][k] = sum_x in[r][x] F[x][k],   rows r = (pol, a): 4 N~ rows; K = N = N~ complex.
+// As a real product (K rows 2x, 2x+1 = re, im of in[.][x]; N columns 2k, 2k+1 = re, im of out[.][k]) it
+// is (N~/4) x (N~/4) tiles of mma.m16n8k16 with N~/8 k-steps, split-f16 (hi*hi + hi*lo + lo*hi, fp32
+// accumulation) like the contraction; the input is scaled by a power of two into f16 range.  Per
+// output and pass this replaces N~ complex MACs on the CUDA cores (2 LDS + 4 FFMA each).
+// ------------------------------------------------------------------------------------------------
+// B fragments of F: entry (k-step ks, n-tile nt, lane (g, q)) = {hi, hi, lo, lo} of
+// (B[2x][n], B[2x+1][n]) for x = 8 ks + q and x + 4, n = 8 nt + g, with B[2x][2k] = Re F,
+// B[2x+1][2k] = -Im F, B[2x][2k+1] = Im F, B[2x+1][2k+1] = Re F.  N~^2 entries (16 N~^2 bytes).
+template <int NS>
+__device__ __forceinline__ void dft_btable(uint4 *tab, float sign) {
+    constexpr int NTL = NS / 4, KST = NS / 8, h = NS / 2;
+    for (int e = threadIdx.x; e < KST * NTL * 32; e += blockDim.x) {
+        const int ln = e & 31, t = e >> 5, ks = t / NTL, nt = t - ks * NTL;
+        const int gg = ln >> 2, qq = ln & 3;
+        const int k = nt * 4 + (gg >> 1), im = gg & 1;
+        uint32_t hi[2], lo[2];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            const int x = ks * 8 + qq + 4 * r;
+            int ex = ((k - h) * (x - h)) % NS;
+            ex += ex < 0 ? NS : 0;
+            float sn, cs;
+            sincospif(float(2 * ex) / float(NS), &sn, &cs);
+            sn *= sign;
+            split2(im ? sn : cs, im ? cs : -sn, hi[r], lo[r]);
+        }
+        tab[e] = make_uint4(hi[0], hi[1], lo[0], lo[1]);
+    }
+}
+
+// One pass: in[r][x] = src[pol * N~^2 + a * RS + x * KS] for r = pol N~ + a, multiplied by `scale`
+// (power of two: f16 range); emit(pol, a, k, out[r][k] * outmul) for every output.  Warps take 16x8
+// output tiles round robin.
+template <int NS, int WARPS, typename Emit>
+__device__ __forceinline__ void dft_pass_tc(const float2 *src, int RS, int KS, const uint4 *tab, float scale,
+                                            float outmul, Emit emit) {
+    constexpr int NPIX = NS * NS;
+    constexpr int MTL = NS / 4, NTL = NS / 4, KST = NS / 8;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
+    for (int tile = warp; tile < MTL * NTL; tile += WARPS) {
+        const int mt = tile / NTL, nt = tile - mt * NTL;
+        const int r0 = mt * 16 + g, r1 = r0 + 8;
+        const int p0 = r0 / NS, a0 = r0 - p0 * NS, p1 = r1 / NS, a1 = r1 - p1 * NS;
+        const float2 *s0 = src + p0 * NPIX + a0 * RS, *s1 = src + p1 * NPIX + a1 * RS;
+        float d[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+#pragma unroll
+        for (int ks = 0; ks < KST; ++ks) {
+            const int x = ks * 8 + q;
+            const float2 v00 = s0[x * KS], v10 = s1[x * KS], v01 = s0[(x + 4) * KS], v11 = s1[(x + 4) * KS];
+            uint32_t ah[4], al[4];
+            split2(v00.x * scale, v00.y * scale, ah[0], al[0]);   // A[g][2q..2q+1]
+            split2(v10.x * scale, v10.y * scale, ah[1], al[1]);   // A[g+8][2q..2q+1]
+            split2(v01.x * scale, v01.y * scale, ah[2], al[2]);   // A[g][2q+8..2q+9]
+            split2(v11.x * scale, v11.y * scale, ah[3], al[3]);   // A[g+8][2q+8..2q+9]
+            const uint4 b = tab[(ks * NTL + nt) * 32 + lane];
+            mma16816(d, ah[0], ah[1], ah[2], ah[3], b.x, b.y);
+            mma16816(d, ah[0], ah[1], ah[2], ah[3], b.z, b.w);
+            mma16816(d, al[0], al[1], al[2], al[3], b.x, b.y);
+        }
+        const int k = nt * 4 + q;
+        emit(p0, a0, k, make_float2(d[0] * outmul, d[1] * outmul));
+        emit(p1, a1, k, make_float2(d[2] * outmul, d[3] * outmul));
+    }
+}
+
+// a3 + a4 + a5 with the tensor-core DFT.  On entry (after a barrier) sub_s[pol][pix] holds the raw
+// image-domain sums of the item; tmp_s holds 4 N~^2 complex, tab 16 N~^2 bytes.
+template <int NS, int WARPS>
+__device__ __forceinline__ void gridder_epilogue_tc(const KernelArgs &a, const ItemSetup &s, float2 *sub_s,
+                                                    float2 *tmp_s, uint4 *tab, float *red_s) {
+    constexpr int NPIX = NS * NS;
+    const idg_metadata &md = s.md;
+    float mx = 0.0f;
+    for (int pix = threadIdx.x; pix < NPIX; pix += WARPS * 32)
+        mx = fmaxf(mx, dev::gridder_aterm_pixel<NS>(a, s, sub_s, pix));     // a3
+    dft_btable<NS>(tab, -1.0f);
+    const float sc = pow2_scale(block_max<WARPS>(mx, red_s));  // (its barriers publish sub_s and tab)
+    // a4 rows: T[pol][y][kx] -> tmp_s[pol][kx][y], kept scaled by sc / 32 (|T| <= N~ max|S|)
+    dft_pass_tc<NS, WARPS>(sub_s, NS, 1, tab, sc, 1.0f / 32.0f, [&](int pol, int y, int kx, float2 v) {
+        tmp_s[pol * NPIX + kx * NS + y] = v;
+    });
+    __syncthreads();
+    // a4 columns + a5: G[pol][ky][kx] = sum_y T[pol][y][kx] F[y][ky], added to the grid
+    const int64_t gs = a.grid_size;
+    float2 *gp = a.grid + (int64_t(md.z) * 4 * gs + md.y) * gs + md.x;
+    dft_pass_tc<NS, WARPS>(tmp_s, NS, 1, tab, 1.0f, 32.0f / sc, [&](int pol, int kx, int ky, float2 v) {
+        dev::red_add(gp + (int64_t(pol) * gs + ky) * gs + kx, v);
+    });
+}
+
+// a6 + a7 with the tensor-core DFT: splitter (grid -> sub_s), centred inverse DFT (columns, then rows);
+// on return (after a barrier) sub_s[pol][y][x] holds the image-domain subgrid before a8.  tab is
+// 16 N~^2 bytes of scratch (dead on return).
+template <int NS, int WARPS>
+__device__ __forceinline__ void degridder_prologue_tc(const KernelArgs &a, const ItemSetup &s, float2 *sub_s,
+                                                      float2 *tmp_s, uint4 *tab, float *red_s) {
+    constexpr int NPIX = NS * NS;
+    constexpr int NT = WARPS * 32;
+    constexpr int PER = (4 * NPIX + NT - 1) / NT;
+    const idg_metadata &md = s.md;
+    const int64_t gs = a.grid_size;
+    const float2 *gp = a.grid + (int64_t(md.z) * 4 * gs + md.y) * gs + md.x;
+    float2 v[PER];
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {   // a6: all loads in flight before any use
+        const int o = threadIdx.x + i * NT;
+        if (o < 4 * NPIX) {
+            const int pol = o / NPIX, rem = o - pol * NPIX, ky = rem / NS, kx = rem - ky * NS;
+            v[i] = gp[(int64_t(pol) * gs + ky) * gs + kx];
+        }
+    }
+    dft_btable<NS>(tab, +1.0f);
+    float mx = 0.0f;
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {
+        const int o = threadIdx.x + i * NT;
+        if (o < 4 * NPIX) {
+            sub_s[o] = v[i];
+            mx = fmaxf(mx, fmaxf(fabsf(v[i].x), fabsf(v[i].y)));
+        }
+    }
+    const float sc = pow2_scale(block_max<WARPS>(mx, red_s));  // (its barriers publish sub_s and tab)
+    // a7 columns: rows (pol, kx), K = ky -> tmp_s[pol][y][kx], kept scaled by sc / 32
+    dft_pass_tc<NS, WARPS>(sub_s, 1, NS, tab, sc, 1.0f / 32.0f, [&](int pol, int kx, int y, float2 w) {
+        tmp_s[pol * NPIX + y * NS + kx] = w;
+    });
+    __syncthreads();
+    // a7 rows: rows (pol, y), K = kx -> sub_s[pol][y][x]
+    dft_pass_tc<NS, WARPS>(tmp_s, NS, 1, tab, 1.0f, 32.0f / sc, [&](int pol, int y, int x, float2 w) {
+        sub_s[pol * NPIX + y * NS + x] = w;
+    });
+    __syncthreads();
+}
+
+// ------------------------------------------------------------------------------------------------
 // Tensor-core gridder.  One CTA per work item; WARPS warps x MT m-tiles x 16 pixels = N~^2.
 // k-block = 8 visibilities = 8 consecutive channels of one timestep (requires C~ % 8 == 0).
 // ------------------------------------------------------------------------------------------------
@@ -138,7 +276,7 @@ inline size_t gridder_tc_smem_bytes(int NS, int max_channels, int kbb_ = kTcBatc
     const size_t kbb = kbb_;
     const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + kbb * 4 * 16 /*df*/ +
                         (kbb + 1) * 32 /*coef*/ + size_t(max_channels) * 4;
-    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2);
+    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2) + size_t(NS) * NS * 16;  // sub, tmp, DFT table
     return std::max(main, epi) + 16;
 }
 
@@ -160,7 +298,6 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
     float4 *coef_s = reinterpret_cast<float4 *>(dfk_s + KBB * 4);    // [KBB+1][2]
     float *df_s = reinterpret_cast<float *>(coef_s + 2 * (KBB + 1)); // [nc]
     __shared__ float red_s[WARPS];
-    __shared__ float2 tw[NS];
 
     const int item = a.order[blockIdx.x];
     const ItemSetup s = dev::item_setup(a, item, NS);
@@ -333,7 +470,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
         sub_s[q * NPIX + p0 + 8] = make_float2(acc[i][2] * inv, acc[i][3] * inv);
     }
     __syncthreads();
-    dev::gridder_epilogue<NS>(a, s, sub_s, tmp_s, tw);
+    gridder_epilogue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(tmp_s + 4 * NPIX), red_s);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -353,7 +490,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
 inline size_t gridder_rot_smem_bytes(int NS, int kbb_ = kTcBatchKB) {
     const size_t kbb = kbb_;
     const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + (kbb + 1) * 32 /*coef*/;
-    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2);
+    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2) + size_t(NS) * NS * 16;  // sub, tmp, DFT table
     return std::max(main, epi) + 16;
 }
 
@@ -371,7 +508,6 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot_kernel(const Ker
     uint4 *frag_s = reinterpret_cast<uint4 *>(raw_s + 2 * VB);       // [KBB][32]
     float4 *coef_s = reinterpret_cast<float4 *>(frag_s + KBB * 32);  // [KBB+1][2]
     __shared__ float red_s[WARPS];
-    __shared__ float2 tw[NS];
 
     const int item = a.order[blockIdx.x];
     const ItemSetup s = dev::item_setup(a, item, NS);
@@ -526,7 +662,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot_kernel(const Ker
         sub_s[q * NPIX + p0 + 8] = make_float2(acc[i][2] * inv, acc[i][3] * inv);
     }
     __syncthreads();
-    dev::gridder_epilogue<NS>(a, s, sub_s, tmp_s, tw);
+    gridder_epilogue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(tmp_s + 4 * NPIX), red_s);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -556,7 +692,6 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     float4 *bq_s = lmn_s + NKB * 8;                                       // [T~][2]: B_t, Q_t of the item
     float *df_s = reinterpret_cast<float *>(bq_s + 2 * a.max_timesteps_in_item);  // [C~]: nu/c - f_ref
     __shared__ float red_s[WARPS];
-    __shared__ float2 tw[NS];
 
     const int item = a.order[blockIdx.x];
     const ItemSetup s = dev::item_setup(a, item, NS);
@@ -575,14 +710,16 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     }
     for (int c = threadIdx.x; c < nc; c += NT)
         df_s[c] = float(a.frequencies[md.channel_begin + c] / kSpeedOfLight - s.f_ref);
-    dev::degridder_split_columns<NS>(a, s, sub_s, tmp_s, tw);  // (its barriers publish bq_s / df_s)
+    // a6 + a7 (tensor-core DFT; the table aliases lmn_s, written only after it)
+    degridder_prologue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(lmn_s), red_s);
     float2 rr[PPT][4];
     float mx = 0.0f;
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
         const int pix = threadIdx.x + i * NT;
         if (pix < NPIX) {
-            dev::degridder_pixel<NS>(a, s, tmp_s, tw, pix, rr[i]);
+            const float2 sv[4] = {sub_s[pix], sub_s[NPIX + pix], sub_s[2 * NPIX + pix], sub_s[3 * NPIX + pix]};
+            dev::degridder_aterm_pixel<NS>(a, s, sv, pix, rr[i]);   // a8
 #pragma unroll
             for (int p = 0; p < 4; ++p) mx = fmaxf(mx, fmaxf(fabsf(rr[i][p].x), fabsf(rr[i][p].y)));
             const int y = pix / NS, x = pix - y * NS;
