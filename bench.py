@@ -194,6 +194,19 @@ def run_reference(args):
 # ------------------------------------------------------------------------------------------------
 # our arm
 # ------------------------------------------------------------------------------------------------
+def sincos_per_pair(variant: str, nc_item: int) -> float:
+    """sincos evaluations per (pixel, visibility) pair of a kernel variant (the paper's kernels and
+    the direct tensor-core kernels: 1).  gridder_rot: per (pixel, timestep) 8 slot phasors + E_t in each
+    of the 4 lanes sharing the pixel, for 8 J pairs (J = channel groups of 8); gridder_tcr: half the
+    phasors by recurrence plus one step phasor per (pixel, timestep) in each of the 2 lanes."""
+    j = max(1, nc_item // 8)
+    if variant.startswith("gridder_rot"):
+        return (8.0 + (4.0 if j > 1 else 0.0)) / (8.0 * j)
+    if variant.startswith("gridder_tcr"):
+        return 0.5 + 0.5 / j
+    return 1.0
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -369,15 +382,21 @@ def run_ours(args):
         for r in (0, 1, 2, 4, 8, 12, 16, 17, 24, 32, 64):
             rho_sweep[str(r)] = best(r, args.rho_iterations) / 1e12
     per_kernel = {}
+    md = plan.metadata()
+    nc_item = int((md["channel_end"] - md["channel_begin"]).max()) if len(md) else 1
     for name in ("gridder", "degridder"):
         k = kern.get(name)
         if not k:
             continue
         avg_ms = k["total_ms"] / k["launches"]
         achieved = OPS_PER_PAIR * pairs / (avg_ms * 1e-3) / 1e12
+        variant = idg.last_variant(name)
+        spp = sincos_per_pair(variant, nc_item)
         per_kernel[name] = {"launches": k["launches"], "avg_ms": avg_ms, "TOps_s": achieved,
                             "frac_xu_sincos": achieved / xu_peak, "frac_rho17": achieved / rho17,
-                            "share_of_step": k["total_ms"] / ms}
+                            "share_of_step": k["total_ms"] / ms, "variant": variant,
+                            "sincos_per_pair": spp, "peak_own_TOps_s": xu_peak / spp,
+                            "frac_own_bound": achieved * spp / xu_peak}
     dominant = max(per_kernel, key=lambda n: per_kernel[n]["avg_ms"]) if per_kernel else None
     sm_mhz = clocks.summary()["sm_mhz"] or 1965
     traffic = None
@@ -393,8 +412,11 @@ def run_ours(args):
                     "peak": xu_peak, "unit": "TOps/s", "frac": per_kernel[dominant]["frac_xu_sincos"],
                     "traffic": traffic,
                     "peak_source": "measured sincos throughput of the XU/MUFU pipe (idg_rho_benchmark rho=0) "
-                                   "x 36 paper-ops per pair, this process; the binding unit of the "
-                                   "tensor-core kernels (1 sincos per pair)",
+                                   "x 36 paper-ops per pair, this process: the sincos roofline of a kernel "
+                                   "that evaluates one sincos per (pixel, visibility) pair (the paper's "
+                                   "kernels, the degridder); kernels['gridder'] reports its own bound "
+                                   "(fewer sincos per pair by accumulator rotation) as peak_own_TOps_s",
+                    "variant": per_kernel[dominant]["variant"],
                     "peak_rho17": rho17, "frac_rho17": per_kernel[dominant]["frac_rho17"],
                     "peak_rho17_source": "paper's modified roofline: FMA:sincos mix at rho=17 (P:276-290), "
                                          "measured in this process",
@@ -414,8 +436,10 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": workload_description(args.config), "visibilities": int(nvis_total),
-                   "arithmetic": "fp32 phases + MUFU sincos; pixel x visibility products on tensor cores as "
-                                 "split-f16 (hi*hi + hi*lo + lo*hi) mma with fp32 accumulation",
+                   "arithmetic": "fp32 phases + MUFU sincos; pixel x visibility products and the subgrid "
+                                 "DFTs on tensor cores as split-f16 (hi*hi + hi*lo + lo*hi) mma with fp32 "
+                                 "accumulation; gridder: phasors of 8 channels per timestep rotated to the "
+                                 "other channel groups on the fp32 accumulators (uniform channels)",
                    "subgrids_rank0": st["nr_subgrids"], "pairs_rank0": pairs,
                    "parallelism": f"baseline shards x{world}" + (" + NCCL reduce/broadcast" if world > 1 else ""),
                    "l2": f"inputs larger than L2 (visibilities {vis_bytes / 1e9:.1f} GB/step)",

@@ -198,6 +198,11 @@ idg_status idg_profiling_read(idg_kernel_time *dst, int32_t capacity, int32_t *n
  * is the fastest eligible tensor-core variant. */
 const char *idg_kernel_variants(int32_t which);
 
+/* Diagnostics: name of the variant (one of idg_kernel_variants(which)) that the most recent gridder
+ * (which = 0) or degridder (which = 1) launch in this process used, or "" before the first launch.
+ * Static storage; safe to call from any thread (the name may be stale if calls race). */
+const char *idg_last_variant(int32_t which);
+
 /* Number of kernel launches issued by this library in the calling process so far. */
 int64_t idg_launch_count(void);
 

@@ -299,6 +299,8 @@ int64_t idg_launch_count(void) { return g_launches.load(); }
 
 const char *idg_kernel_variants(int32_t which) { return idg::variant_names(which == 0 ? 0 : 1); }
 
+const char *idg_last_variant(int32_t which) { return idg::last_variant(which == 0 ? 0 : 1); }
+
 idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, int32_t nr_baselines,
                            int32_t nr_timesteps, int32_t nr_channels, const float *uvw,
                            const double *frequencies, const idg_baseline *baselines,

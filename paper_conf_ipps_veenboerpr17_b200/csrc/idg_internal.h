@@ -74,6 +74,7 @@ const Variant *tf32_degridder_variants(int *n);
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s);
 cudaError_t launch_degridder(const KernelArgs &a, cudaStream_t s);
 const char *variant_names(int which);
+const char *last_variant(int which);   // name of the variant the last launch used ("" before any)
 cudaError_t launch_rho_benchmark(int rho, int iterations, float *d_out, cudaStream_t s,
                                  int *blocks, int *threads, int *units_per_thread);
 

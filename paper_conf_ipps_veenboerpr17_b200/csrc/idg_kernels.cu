@@ -24,6 +24,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstdlib>
 #include <cstring>
 #include <string>
@@ -380,19 +381,27 @@ const std::vector<const Variant *> &tensor_variants(int which) {
 
 }  // namespace
 
+std::atomic<const char *> g_last_variant[2] = {"", ""};
+
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
     const Variant *var = pick(kGridderVariants, int(std::size(kGridderVariants)), tensor_variants(0), a,
                               "IDG_GRIDDER_VARIANT");
-    return var ? var->fn(a, s) : cudaErrorInvalidValue;
+    if (!var) return cudaErrorInvalidValue;
+    g_last_variant[0].store(var->name);
+    return var->fn(a, s);
 }
 
 cudaError_t launch_degridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;
     const Variant *var = pick(kDegridderVariants, int(std::size(kDegridderVariants)), tensor_variants(1), a,
                               "IDG_DEGRIDDER_VARIANT");
-    return var ? var->fn(a, s) : cudaErrorInvalidValue;
+    if (!var) return cudaErrorInvalidValue;
+    g_last_variant[1].store(var->name);
+    return var->fn(a, s);
 }
+
+const char *last_variant(int which) { return g_last_variant[which == 0 ? 0 : 1].load(); }
 
 const char *variant_names(int which) {
     static std::string names[2];

@@ -21,7 +21,10 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdint>
+#include <mutex>
+#include <vector>
 
 #include "idg_device.cuh"
 #include "idg_internal.h"
@@ -139,28 +142,28 @@ __device__ __forceinline__ float4 abs_max4(float4 v, float m) {
 // ------------------------------------------------------------------------------------------------
 // B fragments of F: entry (k-step ks, n-tile nt, lane (g, q)) = {hi, hi, lo, lo} of
 // (B[2x][n], B[2x+1][n]) for x = 8 ks + q and x + 4, n = 8 nt + g, with B[2x][2k] = Re F,
-// B[2x+1][2k] = -Im F, B[2x][2k+1] = Im F, B[2x+1][2k+1] = Re F.  N~^2 entries (16 N~^2 bytes).
+// B[2x+1][2k] = -Im F, B[2x][2k+1] = Im F, B[2x+1][2k+1] = Re F.  N~^2 entries per subgrid size and
+// direction, computed on the host in fp64 once per device (ensure_dft_tables) and read through the
+// read-only cache (9 KB for N~ = 24: L1-resident for every CTA).
+constexpr int kDftTabEntries = 16 * 16 + 24 * 24 + 32 * 32;
+__device__ uint4 g_dft_tab[2][kDftTabEntries];   // [0]: sign -1 (gridding), [1]: sign +1 (degridding)
+__host__ __device__ constexpr int dft_tab_offset(int ns) { return ns == 16 ? 0 : ns == 24 ? 256 : 832; }
 template <int NS>
-__device__ __forceinline__ void dft_btable(uint4 *tab, float sign) {
-    constexpr int NTL = NS / 4, KST = NS / 8, h = NS / 2;
-    for (int e = threadIdx.x; e < KST * NTL * 32; e += blockDim.x) {
-        const int ln = e & 31, t = e >> 5, ks = t / NTL, nt = t - ks * NTL;
-        const int gg = ln >> 2, qq = ln & 3;
-        const int k = nt * 4 + (gg >> 1), im = gg & 1;
-        uint32_t hi[2], lo[2];
-#pragma unroll
-        for (int r = 0; r < 2; ++r) {
-            const int x = ks * 8 + qq + 4 * r;
-            int ex = ((k - h) * (x - h)) % NS;
-            ex += ex < 0 ? NS : 0;
-            float sn, cs;
-            sincospif(float(2 * ex) / float(NS), &sn, &cs);
-            sn *= sign;
-            split2(im ? sn : cs, im ? cs : -sn, hi[r], lo[r]);
-        }
-        tab[e] = make_uint4(hi[0], hi[1], lo[0], lo[1]);
+__device__ __forceinline__ const uint4 *dft_tab(int sign) {
+    return g_dft_tab[sign < 0 ? 0 : 1] + dft_tab_offset(NS);
+}
+
+// Copy the table of one direction into shared memory (cp.async, 16 B per thread-op; completes at the
+// caller's cp.async.wait_all + barrier).
+template <int NS>
+__device__ __forceinline__ void dft_tab_to_smem(uint4 *dst, int sign) {
+    const uint4 *src = dft_tab<NS>(sign);
+    for (int e = threadIdx.x; e < NS * NS; e += blockDim.x) {
+        const unsigned d = static_cast<unsigned>(__cvta_generic_to_shared(dst + e));
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src + e) : "memory");
     }
 }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
 // One pass: in[r][x] = src[pol * N~^2 + a * RS + x * KS] for r = pol N~ + a, multiplied by `scale`
 // (power of two: f16 range); emit(pol, a, k, out[r][k] * outmul) for every output.  Warps take 16x8
@@ -198,16 +201,17 @@ __device__ __forceinline__ void dft_pass_tc(const float2 *src, int RS, int KS, c
 }
 
 // a3 + a4 + a5 with the tensor-core DFT.  On entry (after a barrier) sub_s[pol][pix] holds the raw
-// image-domain sums of the item; tmp_s holds 4 N~^2 complex, tab 16 N~^2 bytes.
+// image-domain sums of the item; tmp_s holds 4 N~^2 complex, tab N~^2 uint4 (the DFT table).
 template <int NS, int WARPS>
 __device__ __forceinline__ void gridder_epilogue_tc(const KernelArgs &a, const ItemSetup &s, float2 *sub_s,
                                                     float2 *tmp_s, uint4 *tab, float *red_s) {
     constexpr int NPIX = NS * NS;
     const idg_metadata &md = s.md;
+    dft_tab_to_smem<NS>(tab, -1);
     float mx = 0.0f;
     for (int pix = threadIdx.x; pix < NPIX; pix += WARPS * 32)
         mx = fmaxf(mx, dev::gridder_aterm_pixel<NS>(a, s, sub_s, pix));     // a3
-    dft_btable<NS>(tab, -1.0f);
+    cp_async_wait_all();
     const float sc = pow2_scale(block_max<WARPS>(mx, red_s));  // (its barriers publish sub_s and tab)
     // a4 rows: T[pol][y][kx] -> tmp_s[pol][kx][y], kept scaled by sc / 32 (|T| <= N~ max|S|)
     dft_pass_tc<NS, WARPS>(sub_s, NS, 1, tab, sc, 1.0f / 32.0f, [&](int pol, int y, int kx, float2 v) {
@@ -223,11 +227,13 @@ __device__ __forceinline__ void gridder_epilogue_tc(const KernelArgs &a, const I
 }
 
 // a6 + a7 with the tensor-core DFT: splitter (grid -> sub_s), centred inverse DFT (columns, then rows);
-// on return (after a barrier) sub_s[pol][y][x] holds the image-domain subgrid before a8.  tab is
-// 16 N~^2 bytes of scratch (dead on return).
-template <int NS, int WARPS>
+// on return (after a barrier) sub_s[pol][y][x] holds the image-domain subgrid before a8; tab is N~^2
+// uint4 of scratch for the DFT table (dead on return).  `overlap()`
+// runs while the splitter's loads are in flight (its shared-memory writes are published by the
+// barriers that follow).
+template <int NS, int WARPS, typename Overlap>
 __device__ __forceinline__ void degridder_prologue_tc(const KernelArgs &a, const ItemSetup &s, float2 *sub_s,
-                                                      float2 *tmp_s, uint4 *tab, float *red_s) {
+                                                      float2 *tmp_s, uint4 *tab, float *red_s, Overlap overlap) {
     constexpr int NPIX = NS * NS;
     constexpr int NT = WARPS * 32;
     constexpr int PER = (4 * NPIX + NT - 1) / NT;
@@ -243,7 +249,8 @@ __device__ __forceinline__ void degridder_prologue_tc(const KernelArgs &a, const
             v[i] = gp[(int64_t(pol) * gs + ky) * gs + kx];
         }
     }
-    dft_btable<NS>(tab, +1.0f);
+    dft_tab_to_smem<NS>(tab, +1);
+    overlap();
     float mx = 0.0f;
 #pragma unroll
     for (int i = 0; i < PER; ++i) {
@@ -253,6 +260,7 @@ __device__ __forceinline__ void degridder_prologue_tc(const KernelArgs &a, const
             mx = fmaxf(mx, fmaxf(fabsf(v[i].x), fabsf(v[i].y)));
         }
     }
+    cp_async_wait_all();
     const float sc = pow2_scale(block_max<WARPS>(mx, red_s));  // (its barriers publish sub_s and tab)
     // a7 columns: rows (pol, kx), K = ky -> tmp_s[pol][y][kx], kept scaled by sc / 32
     dft_pass_tc<NS, WARPS>(sub_s, 1, NS, tab, sc, 1.0f / 32.0f, [&](int pol, int kx, int y, float2 w) {
@@ -276,7 +284,7 @@ inline size_t gridder_tc_smem_bytes(int NS, int max_channels, int kbb_ = kTcBatc
     const size_t kbb = kbb_;
     const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + kbb * 4 * 16 /*df*/ +
                         (kbb + 1) * 32 /*coef*/ + size_t(max_channels) * 4;
-    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2) + size_t(NS) * NS * 16;  // sub, tmp, DFT table
+    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2) + size_t(NS) * NS * 16;  // sub_s, tmp_s, DFT table
     return std::max(main, epi) + 16;
 }
 
@@ -490,7 +498,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
 inline size_t gridder_rot_smem_bytes(int NS, int kbb_ = kTcBatchKB) {
     const size_t kbb = kbb_;
     const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + (kbb + 1) * 32 /*coef*/;
-    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2) + size_t(NS) * NS * 16;  // sub, tmp, DFT table
+    const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2) + size_t(NS) * NS * 16;  // sub_s, tmp_s, DFT table
     return std::max(main, epi) + 16;
 }
 
@@ -702,16 +710,20 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     // per-timestep phase coefficients B_t = 2 pi (uvw_t f_ref - uvw0), Q_t = 2 pi uvw_t (fp64 -> fp32,
     // once per item) and channel offsets df_c = nu_c/c - f_ref: a visibility's coefficients are then
     // B_t + df_c Q_t (fp32 FMAs, as in the gridder), with no fp64 work in front of each tile
-    for (int t = threadIdx.x; t < md.nr_timesteps; t += NT) {
-        float4 cB, cQ;
-        dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
-        bq_s[2 * t] = cB;
-        bq_s[2 * t + 1] = cQ;
-    }
-    for (int c = threadIdx.x; c < nc; c += NT)
-        df_s[c] = float(a.frequencies[md.channel_begin + c] / kSpeedOfLight - s.f_ref);
-    // a6 + a7 (tensor-core DFT; the table aliases lmn_s, written only after it)
-    degridder_prologue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(lmn_s), red_s);
+    // (computed while the splitter's loads of a6 are in flight)
+    auto coefficients = [&] {
+        for (int t = threadIdx.x; t < md.nr_timesteps; t += NT) {
+            float4 cB, cQ;
+            dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
+            bq_s[2 * t] = cB;
+            bq_s[2 * t + 1] = cQ;
+        }
+        for (int c = threadIdx.x; c < nc; c += NT)
+            df_s[c] = float(a.frequencies[md.channel_begin + c] / kSpeedOfLight - s.f_ref);
+    };
+    coefficients();
+    // a6 + a7 (tensor-core DFT; its table aliases lmn_s, written only after it)
+    degridder_prologue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(lmn_s), red_s, [] {});
     float2 rr[PPT][4];
     float mx = 0.0f;
 #pragma unroll
@@ -830,8 +842,61 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     }
 }
 
+// Host: the DFT B-fragment tables of g_dft_tab (fp64 cos/sin, split into f16 hi + lo), uploaded once per
+// device before the first tensor-core gridder / degridder launch on it.
+uint32_t h2_pack(double x, double y, bool low_part) {
+    auto part = [&](double v) {
+        const __half hi = __float2half_rn(float(v));
+        const __half h = low_part ? __float2half_rn(float(v - double(__half2float(hi)))) : hi;
+        return uint32_t(__half_raw(h).x);
+    };
+    return part(x) | (part(y) << 16);
+}
+
+cudaError_t ensure_dft_tables() {
+    static std::mutex mu;
+    static std::vector<char> done;
+    int dev = 0;
+    cudaError_t err = cudaGetDevice(&dev);
+    if (err != cudaSuccess) return err;
+    std::lock_guard<std::mutex> lock(mu);
+    if (size_t(dev) < done.size() && done[dev]) return cudaSuccess;
+    std::vector<uint4> tab(2 * size_t(kDftTabEntries));
+    for (int sgn = 0; sgn < 2; ++sgn) {
+        const double sign = sgn == 0 ? -1.0 : 1.0;
+        for (int ns : {16, 24, 32}) {
+            const int ntl = ns / 4, kst = ns / 8, h = ns / 2;
+            for (int e = 0; e < kst * ntl * 32; ++e) {
+                const int ln = e & 31, t = e >> 5, ks = t / ntl, nt = t - ks * ntl;
+                const int gg = ln >> 2, qq = ln & 3;
+                const int k = nt * 4 + (gg >> 1), im = gg & 1;
+                double bx[2], by[2];
+                for (int r = 0; r < 2; ++r) {
+                    const int x = ks * 8 + qq + 4 * r;
+                    int ex = ((k - h) * (x - h)) % ns;
+                    ex += ex < 0 ? ns : 0;
+                    const double ang = 2.0 * 3.14159265358979323846 * double(ex) / double(ns);
+                    const double cs = std::cos(ang), sn = sign * std::sin(ang);
+                    bx[r] = im ? sn : cs;
+                    by[r] = im ? cs : -sn;
+                }
+                tab[size_t(sgn) * kDftTabEntries + dft_tab_offset(ns) + e] =
+                    make_uint4(h2_pack(bx[0], by[0], false), h2_pack(bx[1], by[1], false),
+                               h2_pack(bx[0], by[0], true), h2_pack(bx[1], by[1], true));
+            }
+        }
+    }
+    err = cudaMemcpyToSymbol(g_dft_tab, tab.data(), tab.size() * sizeof(uint4));
+    if (err != cudaSuccess) return err;
+    if (done.size() <= size_t(dev)) done.resize(size_t(dev) + 1, 0);
+    done[dev] = 1;
+    return cudaSuccess;
+}
+
 template <int NS, int WARPS, int MT, int MINB, int REC, int KBB = kTcBatchKB>
 cudaError_t launch_gridder_tc(const KernelArgs &a, cudaStream_t st) {
+    cudaError_t terr = ensure_dft_tables();
+    if (terr != cudaSuccess) return terr;
     const size_t smem = gridder_tc_smem_bytes(NS, a.max_channels_in_item, KBB);
     cudaError_t err = dev::prepare(gridder_tc_kernel<NS, WARPS, MT, MINB, REC, KBB>, smem);
     if (err != cudaSuccess) return err;
@@ -842,6 +907,8 @@ cudaError_t launch_gridder_tc(const KernelArgs &a, cudaStream_t st) {
 
 template <int NS, int WARPS, int MT, int MINB, int KPT, int KBB = kTcBatchKB>
 cudaError_t launch_gridder_rot(const KernelArgs &a, cudaStream_t st) {
+    cudaError_t terr = ensure_dft_tables();
+    if (terr != cudaSuccess) return terr;
     const size_t smem = gridder_rot_smem_bytes(NS, KBB);
     cudaError_t err = dev::prepare(gridder_rot_kernel<NS, WARPS, MT, MINB, KPT, KBB>, smem);
     if (err != cudaSuccess) return err;
@@ -852,6 +919,8 @@ cudaError_t launch_gridder_rot(const KernelArgs &a, cudaStream_t st) {
 
 template <int NS, int WARPS, int MT, int MINB>
 cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
+    cudaError_t terr = ensure_dft_tables();
+    if (terr != cudaSuccess) return terr;
     const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
     cudaError_t err = dev::prepare(degridder_tc_kernel<NS, WARPS, MT, MINB>, smem);
     if (err != cudaSuccess) return err;

@@ -47,7 +47,7 @@ EXPORTED = ["idg_plan_create", "idg_plan_destroy", "idg_plan_nr_subgrids", "idg_
             "idg_plan_stats", "idg_workspace_size", "idg_grid", "idg_degrid", "idg_rho_benchmark",
             "idg_profiling_enable", "idg_profiling_reset", "idg_profiling_read", "idg_launch_count",
             "idg_kernel_variants", "idg_host_workspace_size", "idg_grid_host", "idg_degrid_host",
-            "idg_status_string", "idg_last_error"]
+            "idg_status_string", "idg_last_error", "idg_last_variant"]
 
 
 def lib() -> ctypes.CDLL:
@@ -79,11 +79,14 @@ def lib() -> ctypes.CDLL:
     L.idg_launch_count.restype = i64
     L.idg_kernel_variants.restype = ctypes.c_char_p
     L.idg_kernel_variants.argtypes = [i32]
+    L.idg_last_variant.restype = ctypes.c_char_p
+    L.idg_last_variant.argtypes = [i32]
     L.idg_status_string.restype = ctypes.c_char_p
     L.idg_status_string.argtypes = [i32]
     L.idg_last_error.restype = ctypes.c_char_p
     for f in EXPORTED:
-        if f not in ("idg_launch_count", "idg_status_string", "idg_last_error", "idg_kernel_variants"):
+        if f not in ("idg_launch_count", "idg_status_string", "idg_last_error", "idg_kernel_variants",
+                     "idg_last_variant"):
             getattr(L, f).restype = i32
     _lib = L
     return L
@@ -322,6 +325,11 @@ def profiling_read() -> dict:
 def kernel_variants(which: str) -> list[str]:
     """Compiled launch-shape variants of the 'gridder' or 'degridder' (see IDG_*_VARIANT)."""
     return lib().idg_kernel_variants(0 if which == "gridder" else 1).decode().split()
+
+
+def last_variant(which: str) -> str:
+    """Variant the most recent 'gridder' / 'degridder' launch in this process used ('' before any)."""
+    return lib().idg_last_variant(0 if which == "gridder" else 1).decode()
 
 
 def launch_count() -> int:
