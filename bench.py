@@ -198,12 +198,15 @@ def sincos_per_pair(variant: str, nc_item: int) -> float:
     """sincos evaluations per (pixel, visibility) pair of a kernel variant (the paper's kernels and
     the direct tensor-core kernels: 1).  gridder_rot: per (pixel, timestep) 8 slot phasors + E_t in each
     of the 4 lanes sharing the pixel, for 8 J pairs (J = channel groups of 8); gridder_tcr: half the
-    phasors by recurrence plus one step phasor per (pixel, timestep) in each of the 2 lanes."""
+    phasors by recurrence plus one step phasor per (pixel, timestep) in each of the 2 lanes;
+    degridder_rot: per (visibility row 0, pixel) one phasor and one rotation E for four channel rows."""
     j = max(1, nc_item // 8)
     if variant.startswith("gridder_rot"):
         return (8.0 + (4.0 if j > 1 else 0.0)) / (8.0 * j)
     if variant.startswith("gridder_tcr"):
         return 0.5 + 0.5 / j
+    if variant.startswith("degridder_rot"):
+        return 0.5     # per pixel slot: row 0 and E_tp for 4 channel rows
     return 1.0
 
 
@@ -222,7 +225,8 @@ def run_ours(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
 
-    full = idgsynth.make_observation(args.config)
+    over = {"T": args.timesteps} if args.timesteps else {}
+    full = idgsynth.make_observation(args.config, **over)
     b0, b1 = parallel.shard_range(full.nr_baselines, rank, world)
     obs = full.subset(nr_baselines=b1 - b0, baseline_begin=b0)
     t0 = time.perf_counter()
@@ -435,7 +439,8 @@ def run_ours(args):
         "metric": METRIC, "value": value, "unit": "MVis/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": workload_description(args.config), "visibilities": int(nvis_total),
+        "config": {"workload": workload_description(args.config) + (f" [T reduced to {args.timesteps}]" if args.timesteps else ""),
+                   "visibilities": int(nvis_total),
                    "arithmetic": "fp32 phases + MUFU sincos; pixel x visibility products and the subgrid "
                                  "DFTs on tensor cores as split-f16 (hi*hi + hi*lo + lo*hi) mma with fp32 "
                                  "accumulation; gridder: phasors of 8 channels per timestep rotated to the "
@@ -470,6 +475,8 @@ def main():
     ap.add_argument("--reference-step-s", type=float, default=8.0)
     ap.add_argument("--rho-iterations", type=int, default=16384)
     ap.add_argument("--rho-sweep", action="store_true")
+    ap.add_argument("--timesteps", type=int, default=0,
+                    help="tuning only: override the config's T (the line then names the reduced workload)")
     args = ap.parse_args()
     if args.warmup < 3:
         log("[bench] warmup < 3 violates the timing rules; using 3")

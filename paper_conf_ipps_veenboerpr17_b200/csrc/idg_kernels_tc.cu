@@ -684,53 +684,57 @@ inline size_t degridder_tc_smem_bytes(int NS, int max_timesteps, int max_channel
            size_t(max_timesteps) * 32 /*B_t, Q_t of the item's timesteps*/ + size_t(max_channels) * 4 /*df*/ + 16;
 }
 
-template <int NS, int WARPS, int MT, int MINB>
-__global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const KernelArgs a) {
+// Shared-memory layout of the tensor-core degridders (bytes: degridder_tc_smem_bytes).
+template <int NS>
+struct DegridSmem {
+    static constexpr int NPIX = NS * NS, NKB = NPIX / 8;
+    float2 *sub_s, *tmp_s;   // [4][NS][NS] each (prologue)
+    uint4 *frag_s;           // [NKB][32] B fragments (after the prologue; aliases sub_s / tmp_s)
+    float4 *lmn_s;           // [NKB][4][2] slot pairs {l_q, l_q4, m_q, m_q4}, {n_q, n_q4, 0, 0}
+    float4 *bq_s;            // [T~][2]: B_t, Q_t of the item
+    float *df_s;             // [C~]: nu/c - f_ref
+    __device__ DegridSmem(unsigned char *smem, int max_timesteps) {
+        sub_s = reinterpret_cast<float2 *>(smem);
+        tmp_s = sub_s + 4 * NPIX;
+        frag_s = reinterpret_cast<uint4 *>(smem);
+        lmn_s = reinterpret_cast<float4 *>(smem + size_t(NPIX) * 64);
+        bq_s = lmn_s + NKB * 8;
+        df_s = reinterpret_cast<float *>(bq_s + 2 * max_timesteps);
+    }
+};
+
+// Degridder prologue shared by the tensor-core degridders: per-timestep phase coefficients, a6 + a7
+// (tensor-core DFT), a8 per pixel, and the corrected subgrid as split B fragments (k-block = 8 pixels)
+// + per-pixel {l, m, n}.  Ends with a barrier; returns 1 / (the power-of-two f16 range scale).
+template <int NS, int WARPS>
+__device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const ItemSetup &s, const DegridSmem<NS> &sm,
+                                                    float *red_s) {
     constexpr int NT = WARPS * 32;
     constexpr int NPIX = NS * NS;
-    constexpr int NKB = NPIX / 8;
     constexpr int PPT = (NPIX + NT - 1) / NT;
     constexpr int h = NS / 2;
-    static_assert(NPIX % 8 == 0, "pixels per k-block");
-    extern __shared__ __align__(16) unsigned char smem[];
-    float2 *sub_s = reinterpret_cast<float2 *>(smem);                     // [4][NS][NS]
-    float2 *tmp_s = sub_s + 4 * NPIX;                                     // [4][NS][NS]
-    uint4 *frag_s = reinterpret_cast<uint4 *>(smem);                      // [NKB][32] (after prologue)
-    float4 *lmn_s = reinterpret_cast<float4 *>(smem + size_t(NPIX) * 64); // [NKB][4][2] slot pairs
-    float4 *bq_s = lmn_s + NKB * 8;                                       // [T~][2]: B_t, Q_t of the item
-    float *df_s = reinterpret_cast<float *>(bq_s + 2 * a.max_timesteps_in_item);  // [C~]: nu/c - f_ref
-    __shared__ float red_s[WARPS];
-
-    const int item = a.order[blockIdx.x];
-    const ItemSetup s = dev::item_setup(a, item, NS);
     const idg_metadata &md = s.md;
     const int nc = s.nc;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
-
     // per-timestep phase coefficients B_t = 2 pi (uvw_t f_ref - uvw0), Q_t = 2 pi uvw_t (fp64 -> fp32,
     // once per item) and channel offsets df_c = nu_c/c - f_ref: a visibility's coefficients are then
     // B_t + df_c Q_t (fp32 FMAs, as in the gridder), with no fp64 work in front of each tile
-    // (computed while the splitter's loads of a6 are in flight)
-    auto coefficients = [&] {
-        for (int t = threadIdx.x; t < md.nr_timesteps; t += NT) {
-            float4 cB, cQ;
-            dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
-            bq_s[2 * t] = cB;
-            bq_s[2 * t + 1] = cQ;
-        }
-        for (int c = threadIdx.x; c < nc; c += NT)
-            df_s[c] = float(a.frequencies[md.channel_begin + c] / kSpeedOfLight - s.f_ref);
-    };
-    coefficients();
+    for (int t = threadIdx.x; t < md.nr_timesteps; t += NT) {
+        float4 cB, cQ;
+        dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
+        sm.bq_s[2 * t] = cB;
+        sm.bq_s[2 * t + 1] = cQ;
+    }
+    for (int c = threadIdx.x; c < nc; c += NT)
+        sm.df_s[c] = float(a.frequencies[md.channel_begin + c] / kSpeedOfLight - s.f_ref);
     // a6 + a7 (tensor-core DFT; its table aliases lmn_s, written only after it)
-    degridder_prologue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(lmn_s), red_s, [] {});
+    degridder_prologue_tc<NS, WARPS>(a, s, sm.sub_s, sm.tmp_s, reinterpret_cast<uint4 *>(sm.lmn_s), red_s, [] {});
     float2 rr[PPT][4];
     float mx = 0.0f;
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
         const int pix = threadIdx.x + i * NT;
         if (pix < NPIX) {
-            const float2 sv[4] = {sub_s[pix], sub_s[NPIX + pix], sub_s[2 * NPIX + pix], sub_s[3 * NPIX + pix]};
+            const float2 sv[4] = {sm.sub_s[pix], sm.sub_s[NPIX + pix], sm.sub_s[2 * NPIX + pix], sm.sub_s[3 * NPIX + pix]};
             dev::degridder_aterm_pixel<NS>(a, s, sv, pix, rr[i]);   // a8
 #pragma unroll
             for (int p = 0; p < 4; ++p) mx = fmaxf(mx, fmaxf(fabsf(rr[i][p].x), fabsf(rr[i][p].y)));
@@ -738,16 +742,15 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
             const float l = float(x - h) * a.cell_l, m = float(y - h) * a.cell_l;
             // slot pair (q, q+4) of k-block kb: {l_q, l_q4, m_q, m_q4}, {n_q, n_q4, 0, 0}
             const int kb = pix >> 3, slot = pix & 7, half = slot >> 2;
-            float *rec = reinterpret_cast<float *>(lmn_s + (kb * 4 + (slot & 3)) * 2);
+            float *rec = reinterpret_cast<float *>(sm.lmn_s + (kb * 4 + (slot & 3)) * 2);
             rec[half] = l;
             rec[2 + half] = m;
             rec[4 + half] = dev::w_term_n(l, m);
             rec[6 + half] = 0.0f;
         }
     }
-    const float scale = pow2_scale(block_max<WARPS>(mx, red_s));  // barriers: tmp_s reads are done
-    const float inv = 1.0f / scale;
-    uint32_t *frag_w = reinterpret_cast<uint32_t *>(frag_s);
+    const float scale = pow2_scale(block_max<WARPS>(mx, red_s));  // barriers: sub_s reads are done
+    uint32_t *frag_w = reinterpret_cast<uint32_t *>(sm.frag_s);
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
         const int pix = threadIdx.x + i * NT;
@@ -767,12 +770,33 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
         }
     }
     __syncthreads();
+    return __frcp_rn(scale);
+}
+
+template <int NS, int WARPS, int MT, int MINB>
+__global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const KernelArgs a) {
+    constexpr int NPIX = NS * NS;
+    constexpr int NKB = NPIX / 8;
+    static_assert(NPIX % 8 == 0, "pixels per k-block");
+    extern __shared__ __align__(16) unsigned char smem[];
+    const DegridSmem<NS> sm(smem, a.max_timesteps_in_item);
+    const uint4 *frag_s = sm.frag_s;
+    const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
+    const float *df_s = sm.df_s;
+    __shared__ float red_s[WARPS];
+
+    const int item = a.order[blockIdx.x];
+    const ItemSetup s = dev::item_setup(a, item, NS);
+    const idg_metadata &md = s.md;
+    const int nc = s.nc;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
+    const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s);
 
     const int nvis = md.nr_timesteps * nc;
     const int ntiles = (nvis + 15) >> 4;
     // t = v / nc without an integer division: (v + 1/2) / nc is at least 1/(2 nc) away from an integer,
     // and the fp32 quotient's error (v / nc) 2^-23 is smaller for v < 2^22 (else: integer division)
-    const float rnc = 1.0f / float(nc);
+    const float rnc = __frcp_rn(float(nc));
     const bool fdiv = nvis < (1 << 22);
     auto tstep = [&](int v) { return fdiv ? __float2int_rz((float(v) + 0.5f) * rnc) : v / nc; };
     const int64_t row = int64_t(a.nr_channels) * 4;
@@ -839,6 +863,94 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
                 }
             }
         }
+    }
+}
+
+// ------------------------------------------------------------------------------------------------
+// Tensor-core degridder with phasor rotation across channel groups (uniform channels, C~ % 32 == 0).
+// A warp takes 32 channels of one timestep as two m-tiles, so each thread's four A rows are the
+// channels c0 + g + 8r (r = 0..3) of the same timestep.  With the phase linear in frequency,
+//     Phi(t, c + 8r, p) = Phi(t, c, p) E_tp^r,    E_tp = exp(i 8 dnu/c Q_t(p))
+// so per pixel slot the thread evaluates two sincos (row 0 and E) instead of four and forms rows
+// 1..3 by complex products (fp32, on the FMA pipe) before the operand split.  Exact in exact
+// arithmetic; the rounding is that of up to three extra complex products per phasor.
+// ------------------------------------------------------------------------------------------------
+template <int NS, int WARPS, int MINB, int UNR>
+__global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
+    constexpr int NPIX = NS * NS;
+    constexpr int NKB = NPIX / 8;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const DegridSmem<NS> sm(smem, a.max_timesteps_in_item);
+    const uint4 *frag_s = sm.frag_s;
+    const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
+    const float *df_s = sm.df_s;
+    __shared__ float red_s[WARPS];
+
+    const int item = a.order[blockIdx.x];
+    const ItemSetup s = dev::item_setup(a, item, NS);
+    const idg_metadata &md = s.md;
+    const int nc = s.nc;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
+    const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s);
+
+    const int blocks = nc >> 5;                       // 32-channel blocks per timestep
+    const int nblk = md.nr_timesteps * blocks;
+    const float estep = 8.0f * a.channel_step;
+    const int64_t row = int64_t(a.nr_channels) * 4;
+    float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
+                   int64_t(md.channel_begin) * 4;
+    for (int bk = warp; bk < nblk; bk += WARPS) {
+        const int t = bk / blocks, c0 = (bk - t * blocks) * 32;
+        const float4 cB = bq_s[2 * t], cQ = bq_s[2 * t + 1];
+        const float df = df_s[c0 + g];
+        // row 0 (channel c0 + g) coefficients, and the coefficients of the E phase
+        const f2p cu = dup(fmaf(df, cQ.x, cB.x)), cv = dup(fmaf(df, cQ.y, cB.y)), cw = dup(fmaf(df, cQ.z, cB.z));
+        const f2p eu = dup(estep * cQ.x), ev = dup(estep * cQ.y), ew = dup(estep * cQ.z);
+        float acc[2][4];
+#pragma unroll
+        for (int i = 0; i < 2; ++i)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
+        static_assert(NKB % UNR == 0, "k-block unroll");
+#pragma unroll UNR
+        for (int kb = 0; kb < NKB; ++kb) {
+            const uint4 bf = frag_s[kb * 32 + lane];
+            const float4 lm = lmn_s[(kb * 4 + q) * 2], nn = lmn_s[(kb * 4 + q) * 2 + 1];
+            const f2p l2 = pk(lm.x, lm.y), m2 = pk(lm.z, lm.w), n2 = pk(nn.x, nn.y);
+            const float2 p = unpk(fma2(cu, l2, fma2(cv, m2, mul2(cw, n2))));   // row 0 at slots q, q+4
+            const float2 e = unpk(fma2(eu, l2, fma2(ev, m2, mul2(ew, n2))));   // E phase at slots q, q+4
+            float s0, c0q, s1, c1q, es0, ec0, es1, ec1;
+            __sincosf(p.x, &s0, &c0q);
+            __sincosf(p.y, &s1, &c1q);
+            __sincosf(e.x, &es0, &ec0);
+            __sincosf(e.y, &es1, &ec1);
+            // rows r = 0..3 at slots (q, q+4), packed: C = (cos, cos), S = (sin, sin)
+            f2p C = pk(c0q, c1q), S = pk(s0, s1);
+            const f2p EC = pk(ec0, ec1), ES = pk(es0, es1), NES = pk(-es0, -es1);
+            uint32_t ah[2][4], al[2][4];
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                if (r > 0) {
+                    const f2p Cn = fma2(C, EC, mul2(S, NES));
+                    S = fma2(C, ES, mul2(S, EC));
+                    C = Cn;
+                }
+                const float2 cc = unpk(C), ss = unpk(S);
+                // tile r >> 1, row g (r even) / g+8 (r odd): A regs {(row, q), (row+8, q), (row, q+4), (row+8, q+4)}
+                split_phasor(cc.x, ss.x, ah[r >> 1][r & 1], al[r >> 1][r & 1]);
+                split_phasor(cc.y, ss.y, ah[r >> 1][2 + (r & 1)], al[r >> 1][2 + (r & 1)]);
+            }
+#pragma unroll
+            for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
+#pragma unroll
+            for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
+#pragma unroll
+            for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
+        }
+        float2 *vt = vis0 + int64_t(t) * row + int64_t(c0 + g) * 4 + q;
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+            vt[r * 32] = make_float2(acc[r >> 1][2 * (r & 1)] * inv, acc[r >> 1][2 * (r & 1) + 1] * inv);
     }
 }
 
@@ -944,8 +1056,9 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
      launch_gridder_rot<NS, W, MT, MB, KPT, 128>, 8 * KPT}
 const Variant kTcGridder[] = {
     TGROT(24, 12, 3, 2, 4), TGROT(24, 12, 3, 2, 2), TGROT(24, 12, 3, 1, 2), TGROT(24, 12, 3, 1, 4),
-    TGROT(32, 16, 4, 1, 4), TGROT(32, 16, 4, 1, 2), TGROT(32, 8, 8, 1, 4), TGROT(32, 16, 4, 1, 8),
+    TGROT(32, 16, 4, 2, 4), TGROT(32, 16, 4, 1, 4), TGROT(32, 16, 4, 1, 2), TGROT(32, 8, 8, 1, 4), TGROT(32, 16, 4, 1, 8),
     TGROT(16, 8, 2, 2, 2), TGROT(16, 8, 2, 2, 4), TGROT(24, 12, 3, 1, 8),
+    TGROT(32, 32, 2, 1, 4), TGROT(24, 18, 2, 1, 4), TGROT(24, 18, 2, 1, 2),
     TGB(24, 12, 3, 2, 128), TG(24, 12, 3, 2), TG(24, 6, 6, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
     TG(24, 6, 6, 3), TG(24, 9, 4, 3), TG(24, 4, 9, 4),
     TGR(32, 16, 4, 2), TGR(32, 8, 8, 2), TGR(32, 16, 4, 1),
@@ -959,15 +1072,32 @@ const Variant kTcGridder[] = {
 #undef TGR
 #undef TGROT
 #undef TG
+template <int NS, int WARPS, int MINB, int UNR>
+cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
+    cudaError_t terr = ensure_dft_tables();
+    if (terr != cudaSuccess) return terr;
+    const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
+    cudaError_t err = dev::prepare(degridder_rot_kernel<NS, WARPS, MINB, UNR>, smem);
+    if (err != cudaSuccess) return err;
+    LaunchScope scope("degridder", st);
+    degridder_rot_kernel<NS, WARPS, MINB, UNR><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+#define TDROT(NS, W, MB, U) \
+    {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>}
 #define TD(NS, W, MT, MB) \
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>}
 const Variant kTcDegridder[] = {
+    TDROT(32, 16, 1, 2), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
+    TDROT(24, 8, 4, 1), TDROT(24, 8, 3, 1), TDROT(24, 8, 3, 2), TDROT(16, 8, 4, 1),
     TD(24, 8, 2, 4), TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
     TD(24, 4, 2, 6),
     TD(32, 8, 4, 2), TD(32, 4, 4, 3), TD(32, 8, 8, 1), TD(32, 16, 2, 1),
     TD(16, 8, 4, 2), TD(16, 4, 4, 4), TD(16, 8, 2, 3),
 };
 #undef TD
+#undef TDROT
 
 }  // namespace
 

@@ -1,8 +1,9 @@
 #!/bin/bash
 # Bench the LOFAR (or $CFG) step with several gridder variants: bash scripts/sweep_gridder.sh NAME...
 CFG=${CFG:-lofar}
+TS=${TS:-0}
 for V in "$@"; do
   echo "== $V"
-  IDG_GRIDDER_VARIANT="$V" timeout 600 python bench.py --config $CFG --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --rho-iterations 2048 2>/dev/null \
+  IDG_GRIDDER_VARIANT="$V" timeout 600 python bench.py --config $CFG --timesteps $TS --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --rho-iterations 2048 2>/dev/null \
     | python -c "import json,sys; d=json.loads(sys.stdin.read()); k=d['kernels']; print(f\"value {d['value']:.1f} grid {d['grid_mvis_s']:.1f} degrid {d['degrid_mvis_s']:.1f} MVis/s, gridder {k['gridder']['avg_ms']:.2f} ms, clocks {d['clocks']['sm_mhz']}\")"
 done

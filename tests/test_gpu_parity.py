@@ -67,6 +67,8 @@ CASES = [
     ("small_dde", dict(C=24, C_block=8), None, "spheroidal"),       # 3 channel blocks of 8
     ("small_dde", dict(w_planes=4), None, "spheroidal"),            # W-stacking (NEXT-1, R-21)
     ("lofar_dde", dict(T=512, nr_stations=5, w_planes=3), None, "spheroidal"),
+    ("small_dde", dict(C=64), None, "spheroidal"),                   # 2 blocks of 32 channels per timestep
+    ("small_dde", dict(C=40, C_block=24), None, "spheroidal"),      # 24 + 16 channels: rotation J = 3 and 2
 ]
 
 
@@ -74,7 +76,7 @@ KINDS = {
     "default": (None, None),                       # default tensor-core kernels (split-f16 mma)
     "tc": ("tc", "tc"),                            # direct tensor-core kernels (no channel recurrence)
     "rec": ("gridder_tcr<*", "degridder_tc<*"),    # split-f16 gridder with the channel recurrence
-    "rot": ("gridder_rot<*", "degridder_tc<*"),    # split-f16 gridder with accumulator rotation over channel groups
+    "rot": ("gridder_rot<*", "degridder_rot<*"),   # accumulator / phasor rotation over channel groups
     "tf32": ("gridder_tf32*", "degridder_tf32*"),  # split-tf32 tensor-core kernels
     "umma": ("gridder_umma*", "degridder_tc<*"),    # tcgen05 / TMEM gridder
     "simt": ("simt", "simt"),                      # CUDA-core kernels (the paper's structure)
