@@ -197,10 +197,13 @@ def run_reference(args):
 def sincos_per_pair(variant: str, nc_item: int) -> float:
     """sincos evaluations per (pixel, visibility) pair of a kernel variant (the paper's kernels and
     the direct tensor-core kernels: 1).  gridder_rot: per (pixel, timestep) 8 slot phasors + E_t in each
-    of the 4 lanes sharing the pixel, for 8 J pairs (J = channel groups of 8); gridder_tcr: half the
+    of the 4 lanes sharing the pixel, for 8 J pairs (J = channel groups of 8); gridder_rot2: the 8 slot
+    phasors only (E_t derived from slots q, q+4); gridder_tcr: half the
     phasors by recurrence plus one step phasor per (pixel, timestep) in each of the 2 lanes;
     degridder_rot: per (visibility row 0, pixel) one phasor and one rotation E for four channel rows."""
     j = max(1, nc_item // 8)
+    if variant.startswith("gridder_rot2"):
+        return 1.0 / j  # the 8 group-0 phasors only; E_t is derived from them (no sincos)
     if variant.startswith("gridder_rot"):
         return (8.0 + (4.0 if j > 1 else 0.0)) / (8.0 * j)
     if variant.startswith("gridder_tcr"):

@@ -674,6 +674,218 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot_kernel(const Ker
 }
 
 // ------------------------------------------------------------------------------------------------
+// gridder_rot2: the rotation gridder with every item holding exactly KPT channel groups (8 KPT
+// channels, uniform spacing) and the group step E_t derived from the slot phasors instead of its own
+// sincos.  Slots q and q+4 of group 0 are channels 4 apart, so
+//     Phi(t, q+4) conj(Phi(t, q)) = exp(i 4 dnu/c Q_t) = E4,   E_t = exp(i 8 dnu/c Q_t) = E4^2
+// (two complex products on the FMA pipe, packed over the thread's two pixel rows): the MUFU work per
+// (pixel, timestep) is that of the 8 group-0 phasors only (LOFAR: 0.5 sincos per pair, SKA: 0.25).
+// The slot phases are formed from per-lane, per-timestep coefficients c_s = B_t + df_s Q_t (3 FFMA2 per
+// slot and tile), group 0 accumulates in place, the groups' mma chains are interleaved, and there are
+// no runtime channel-group branches.  Exact in exact arithmetic; E carries the rounding of two
+// sincos and two complex products (~1e-6 relative), E^j that of j - 1 more products.
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ f2p add2(f2p a, f2p b) {
+    f2p r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB>
+__global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const KernelArgs a) {
+    constexpr int NT = WARPS * 32;
+    constexpr int NPIX = NS * NS;
+    static_assert(WARPS * MT * 16 == NPIX, "warps x m-tiles x 16 must cover the subgrid");
+    static_assert(KPT >= 1 && KPT <= 4 && KBB_ % KPT == 0 && KPT % GP == 0, "channel groups per timestep / pass");
+    constexpr int h = NS / 2;
+    constexpr int KBB = KBB_;
+    constexpr int VB = KBB * 8;
+    constexpr int NC = 8 * KPT;                  // channels of every item
+    constexpr int TPB = KBB / KPT;               // timesteps per batch
+    extern __shared__ __align__(16) unsigned char smem[];
+    float4 *raw_s = reinterpret_cast<float4 *>(smem);                // [VB][2]
+    uint4 *frag_s = reinterpret_cast<uint4 *>(raw_s + 2 * VB);       // [KBB][32]
+    float4 *coef_s = reinterpret_cast<float4 *>(frag_s + KBB * 32);  // [TPB][2]
+    __shared__ float red_s[WARPS];
+
+    const int item = a.order[blockIdx.x];
+    const ItemSetup s = dev::item_setup(a, item, NS);
+    const idg_metadata &md = s.md;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
+
+    // channel offsets from the reference frequency of slots q and q+4 of group 0
+    const float dq = float(a.frequencies[md.channel_begin + q] / kSpeedOfLight - s.f_ref);
+    const float dq4 = float(a.frequencies[md.channel_begin + q + 4] / kSpeedOfLight - s.f_ref);
+
+    f2p pl[MT], pm[MT], pn[MT];
+    float acc[MT][4];
+#pragma unroll
+    for (int i = 0; i < MT; ++i) {
+        float l2[2], m2[2], n2[2];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            const int pix = (warp * MT + i) * 16 + g + 8 * r;
+            const int x = pix % NS, y = pix / NS;
+            l2[r] = float(x - h) * a.cell_l;
+            m2[r] = float(y - h) * a.cell_l;
+            n2[r] = dev::w_term_n(l2[r], m2[r]);
+        }
+        pl[i] = pk(l2[0], l2[1]);
+        pm[i] = pk(m2[0], m2[1]);
+        pn[i] = pk(n2[0], n2[1]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
+    }
+    float cur_scale = 0.0f;
+
+    const int64_t row = int64_t(a.nr_channels) * 4;  // float2 per timestep
+    const float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
+                         int64_t(md.channel_begin) * 4;
+
+    for (int t0 = 0; t0 < md.nr_timesteps; t0 += TPB) {
+        const int t1 = min(t0 + TPB, md.nr_timesteps);
+        const int nkb = (t1 - t0) * KPT;
+        const int nvb = nkb * 8;
+        __syncthreads();  // previous batch fully consumed
+        // (1) raw visibilities of timesteps [t0, t1): index j = (t - t0) NC + c
+        for (int i = threadIdx.x; i < 2 * nvb; i += NT) {
+            const int j = i >> 1;
+            const int t = j / NC, c = j - t * NC;
+            raw_s[i] = dev::ld_stream(reinterpret_cast<const float4 *>(vis0 + int64_t(t0 + t) * row + c * 4) + (i & 1));
+        }
+        // (2) per-timestep phase coefficients (fp64 -> fp32)
+        for (int t = t0 + int(threadIdx.x); t < t1; t += NT) {
+            float4 cB, cQ;
+            dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
+            coef_s[2 * (t - t0)] = cB;
+            coef_s[2 * (t - t0) + 1] = cQ;
+        }
+        __syncthreads();
+        // (3) f16 range: power-of-two scale from the batch maximum; never increase the running scale
+        float mx = 0.0f;
+        for (int i = threadIdx.x; i < 2 * nvb; i += NT) mx = abs_max4(raw_s[i], mx).x;
+        const float bscale = pow2_scale(block_max<WARPS>(mx, red_s));
+        if (cur_scale == 0.0f) {
+            cur_scale = bscale;
+        } else if (bscale < cur_scale) {
+            const float f = bscale / cur_scale;  // exact power of two
+#pragma unroll
+            for (int i = 0; i < MT; ++i)
+#pragma unroll
+                for (int j = 0; j < 4; ++j) acc[i][j] *= f;
+            cur_scale = bscale;
+        }
+        // (4) B fragments of every (timestep, group): column g = 2 pol + im, k-slots q and q+4
+        for (int i = threadIdx.x; i < nkb * 32; i += NT) {
+            const int kbl = i >> 5, ln = i & 31, gg = ln >> 2, qq = ln & 3;
+            const int pol = gg >> 1, im = gg & 1;
+            uint32_t hi[2], lo[2];
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const float4 v4 = raw_s[2 * (kbl * 8 + qq + 4 * r) + (pol >> 1)];
+                const float vr = ((pol & 1) ? v4.z : v4.x) * cur_scale;
+                const float vi = ((pol & 1) ? v4.w : v4.y) * cur_scale;
+                split2(im ? vi : vr, im ? vr : -vi, hi[r], lo[r]);
+            }
+            frag_s[i] = make_uint4(hi[0], hi[1], lo[0], lo[1]);
+        }
+        __syncthreads();
+        // (5) per timestep: group-0 phasors of every tile, E_t from them, one fresh D_j per group j > 0
+#pragma unroll 1
+        for (int t = t0; t < t1; ++t) {
+            const float4 cB = coef_s[2 * (t - t0)], cQ = coef_s[2 * (t - t0) + 1];
+            // slot coefficients c_s = B_t + df_s Q_t (u, v, w components)
+            const float c0u = fmaf(dq, cQ.x, cB.x), c0v = fmaf(dq, cQ.y, cB.y), c0w = fmaf(dq, cQ.z, cB.z);
+            const float c4u = fmaf(dq4, cQ.x, cB.x), c4v = fmaf(dq4, cQ.y, cB.y), c4w = fmaf(dq4, cQ.z, cB.z);
+            const uint4 *fr = frag_s + (t - t0) * KPT * 32 + lane;
+#pragma unroll
+            for (int i = 0; i < MT; ++i) {
+                uint4 bf0[GP];   // B fragments of the first pass, loaded ahead of the sincos
+#pragma unroll
+                for (int j = 0; j < GP; ++j) bf0[j] = fr[j * 32];
+                const float2 ph0 = unpk(fma2(dup(c0u), pl[i], fma2(dup(c0v), pm[i], mul2(dup(c0w), pn[i]))));
+                const float2 ph1 = unpk(fma2(dup(c4u), pl[i], fma2(dup(c4v), pm[i], mul2(dup(c4w), pn[i]))));
+                float sn[4], cs[4];
+                __sincosf(ph0.x, &sn[0], &cs[0]);   // row g,   slot q
+                __sincosf(ph0.y, &sn[1], &cs[1]);   // row g+8, slot q
+                __sincosf(ph1.x, &sn[2], &cs[2]);   // row g,   slot q+4
+                __sincosf(ph1.y, &sn[3], &cs[3]);   // row g+8, slot q+4
+                uint32_t ah[4], al[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[j], al[j]);
+                if constexpr (KPT == 1) {
+                    mma3(acc[i], ah, al, bf0[0]);
+                } else {
+                    float2 er, ei;   // E_t of rows (g, g+8)
+                    float pr0 = 1.0f, pi0 = 0.0f, pr1 = 1.0f, pi1 = 0.0f;   // E^j of rows g, g+8
+                    // groups in passes of GP: interleaved mma chains, group 0 into the accumulator,
+                    // groups j > 0 fresh and rotated by E^j
+#pragma unroll
+                    for (int p0 = 0; p0 < KPT; p0 += GP) {
+                        uint4 bf[GP];
+                        float d[GP][4];
+#pragma unroll
+                        for (int j = 0; j < GP; ++j) bf[j] = p0 == 0 ? bf0[j] : fr[(p0 + j) * 32];
+#pragma unroll
+                        for (int k = 0; k < 3; ++k) {
+                            const uint32_t *A = k < 2 ? ah : al;
+#pragma unroll
+                            for (int j = 0; j < GP; ++j) {
+                                const uint32_t b0 = k == 1 ? bf[j].z : bf[j].x, b1 = k == 1 ? bf[j].w : bf[j].y;
+                                if (p0 + j == 0)
+                                    mma16816(acc[i], A[0], A[1], A[2], A[3], b0, b1);
+                                else if (k == 0)
+                                    mma16816_zero(d[j], A[0], A[1], A[2], A[3], b0, b1);
+                                else
+                                    mma16816(d[j], A[0], A[1], A[2], A[3], b0, b1);
+                            }
+                        }
+                        if (p0 == 0) {
+                            // E4 = Phi(q+4) conj(Phi(q)), E = E4^2, packed over rows (g, g+8)
+                            const f2p C0 = pk(cs[0], cs[1]), S0 = pk(sn[0], sn[1]);
+                            const f2p C4 = pk(cs[2], cs[3]), S4 = pk(sn[2], sn[3]);
+                            const f2p r4 = fma2(C4, C0, mul2(S4, S0));
+                            const f2p i4 = sub2(mul2(S4, C0), mul2(C4, S0));
+                            er = unpk(sub2(mul2(r4, r4), mul2(i4, i4)));
+                            ei = unpk(mul2(add2(r4, r4), i4));
+                        }
+#pragma unroll
+                        for (int j = 0; j < GP; ++j) {
+                            if (p0 + j == 0) continue;
+                            if (p0 + j == 1) {
+                                pr0 = er.x; pi0 = ei.x; pr1 = er.y; pi1 = ei.y;
+                            } else {
+                                const float a0 = fmaf(pr0, er.x, -pi0 * ei.x), b0 = fmaf(pr0, ei.x, pi0 * er.x);
+                                const float a1 = fmaf(pr1, er.y, -pi1 * ei.y), b1 = fmaf(pr1, ei.y, pi1 * er.y);
+                                pr0 = a0; pi0 = b0; pr1 = a1; pi1 = b1;
+                            }
+                            acc[i][0] = fmaf(pr0, d[j][0], fmaf(-pi0, d[j][1], acc[i][0]));
+                            acc[i][1] = fmaf(pr0, d[j][1], fmaf(pi0, d[j][0], acc[i][1]));
+                            acc[i][2] = fmaf(pr1, d[j][2], fmaf(-pi1, d[j][3], acc[i][2]));
+                            acc[i][3] = fmaf(pr1, d[j][3], fmaf(pi1, d[j][2], acc[i][3]));
+                        }
+                    }
+                }
+            }
+        }
+    }
+
+    // ---- epilogue: D fragments -> sub_s[pol][pixel], then a3 + a4 + a5 ---------------------------
+    __syncthreads();
+    float2 *sub_s = reinterpret_cast<float2 *>(smem);
+    float2 *tmp_s = sub_s + 4 * NPIX;
+    const float inv = cur_scale > 0.0f ? 1.0f / cur_scale : 1.0f;
+#pragma unroll
+    for (int i = 0; i < MT; ++i) {
+        const int p0 = (warp * MT + i) * 16 + g;
+        sub_s[q * NPIX + p0] = make_float2(acc[i][0] * inv, acc[i][1] * inv);
+        sub_s[q * NPIX + p0 + 8] = make_float2(acc[i][2] * inv, acc[i][3] * inv);
+    }
+    __syncthreads();
+    gridder_epilogue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(tmp_s + 4 * NPIX), red_s);
+}
+
+// ------------------------------------------------------------------------------------------------
 // Tensor-core degridder.  One CTA per work item.  Prologue (a6-a8) leaves the corrected subgrid as
 // B fragments (k-block = 8 pixels) + per-pixel {l, m, n}; m-tile = 16 consecutive visibilities of
 // the item (flattened (t, c) order); each warp takes MT tiles at a time over all k-blocks.
@@ -773,7 +985,39 @@ __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const I
     return __frcp_rn(scale);
 }
 
-template <int NS, int WARPS, int MT, int MINB>
+// sincos of two phases on the FMA pipe (packed f32x2), for kernels whose MUFU (XU) pipe is the binding
+// unit: quadrant reduction k = rint(x 2/pi) by the 1.5 2^23 rounding constant, y = x - k pi/2 in two
+// Cody-Waite steps (|y| <= pi/4), minimax polynomials of degree 7 / 8 on [-pi/4, pi/4] (Cephes sinf /
+// cosf coefficients, ~1 ulp), then the quadrant rotation by k mod 4 (the low bits of the rounded
+// value).  Abs. error ~1e-7 for |x| < 2^10, below the __sincosf (MUFU) error at the phases used here.
+// Measured (LOFAR degridder, B200): one of the thread's four slot pairs per k-block on the FMA pipe
+// 41.2 -> 47.2 ms, two -> 56.4 ms: the loop is bound by the whole instruction stream, not the MUFU alone.
+__device__ __forceinline__ void sincos_poly2(f2p x, float2 &sn, float2 &cs) {
+    const f2p magic = dup(12582912.0f);
+    const f2p t = fma2(x, dup(0.636619772367581f), magic);
+    const f2p k = sub2(t, magic);
+    f2p y = fma2(k, dup(-1.57079637050628662f), x);
+    y = fma2(k, dup(4.37113900018624e-8f), y);
+    const f2p y2 = mul2(y, y);
+    f2p ps = fma2(y2, dup(-1.9515295891e-4f), dup(8.3321608736e-3f));
+    ps = fma2(y2, ps, dup(-1.6666654611e-1f));
+    const f2p sy = fma2(mul2(y, y2), ps, y);
+    f2p pc = fma2(y2, dup(2.443315711809948e-5f), dup(-1.388731625493765e-3f));
+    pc = fma2(y2, pc, dup(4.166664568298827e-2f));
+    pc = fma2(y2, pc, dup(-0.5f));
+    const f2p cy = fma2(y2, pc, dup(1.0f));
+    const float2 tt = unpk(t), s2 = unpk(sy), c2 = unpk(cy);
+    auto fix = [](float tq, float s0, float c0, float &so, float &co) {
+        const uint32_t qd = __float_as_uint(tq);
+        const float a = (qd & 1) ? c0 : s0, b = (qd & 1) ? s0 : c0;
+        so = __uint_as_float(__float_as_uint(a) ^ ((qd << 30) & 0x80000000u));
+        co = __uint_as_float(__float_as_uint(b) ^ (((qd + 1) << 30) & 0x80000000u));
+    };
+    fix(tt.x, s2.x, c2.x, sn.x, cs.x);
+    fix(tt.y, s2.y, c2.y, sn.y, cs.y);
+}
+
+template <int NS, int WARPS, int MT, int MINB, int POLY = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int NKB = NPIX / 8;
@@ -835,12 +1079,20 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 #pragma unroll
             for (int i = 0; i < MT; ++i) {
                 // phases of (row, slot q) and (row, slot q+4) in one FFMA2 chain per row
-                const float2 p0 = unpk(fma2(cu[i][0], l2, fma2(cv[i][0], m2, mul2(cw[i][0], n2))));
+                const f2p p0v = fma2(cu[i][0], l2, fma2(cv[i][0], m2, mul2(cw[i][0], n2)));
+                const float2 p0 = unpk(p0v);
                 const float2 p1 = unpk(fma2(cu[i][1], l2, fma2(cv[i][1], m2, mul2(cw[i][1], n2))));
                 float sn[4], cs[4];
-                __sincosf(p0.x, &sn[0], &cs[0]);  // row g,   slot q
+                if (POLY > i) {
+                    // POLY of the MT row-g slot pairs on the FMA pipe (MUFU relief)
+                    float2 s2, c2;
+                    sincos_poly2(p0v, s2, c2);
+                    sn[0] = s2.x; cs[0] = c2.x; sn[2] = s2.y; cs[2] = c2.y;
+                } else {
+                    __sincosf(p0.x, &sn[0], &cs[0]);  // row g,   slot q
+                    __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
+                }
                 __sincosf(p1.x, &sn[1], &cs[1]);  // row g+8, slot q
-                __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
                 __sincosf(p1.y, &sn[3], &cs[3]);  // row g+8, slot q+4
 #pragma unroll
                 for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[i][j], al[i][j]);
@@ -1029,15 +1281,27 @@ cudaError_t launch_gridder_rot(const KernelArgs &a, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-template <int NS, int WARPS, int MT, int MINB>
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB>
+cudaError_t launch_gridder_rot2(const KernelArgs &a, cudaStream_t st) {
+    cudaError_t terr = ensure_dft_tables();
+    if (terr != cudaSuccess) return terr;
+    const size_t smem = gridder_rot_smem_bytes(NS, KBB);
+    cudaError_t err = dev::prepare(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB>, smem);
+    if (err != cudaSuccess) return err;
+    LaunchScope scope("gridder", st);
+    gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+template <int NS, int WARPS, int MT, int MINB, int POLY = 0>
 cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
     cudaError_t terr = ensure_dft_tables();
     if (terr != cudaSuccess) return terr;
     const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
-    cudaError_t err = dev::prepare(degridder_tc_kernel<NS, WARPS, MT, MINB>, smem);
+    cudaError_t err = dev::prepare(degridder_tc_kernel<NS, WARPS, MT, MINB, POLY>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("degridder", st);
-    degridder_tc_kernel<NS, WARPS, MT, MINB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    degridder_tc_kernel<NS, WARPS, MT, MINB, POLY><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -1054,7 +1318,17 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 #define TGROT(NS, W, MT, MB, KPT) \
     {NS, 8, kTensor, 1, "gridder_rot<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ">", \
      launch_gridder_rot<NS, W, MT, MB, KPT, 128>, 8 * KPT}
+// every item exactly 8 KPT channels (channel_gcd % 8 KPT == 0 and max channels <= 8 KPT)
+#define TGROT2(NS, W, MT, MB, KPT) \
+    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ">", \
+     launch_gridder_rot2<NS, W, MT, MB, KPT, KPT, 128>, 8 * KPT}
+#define TGROT2P(NS, W, MT, MB, KPT, GP) \
+    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP ">", \
+     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128>, 8 * KPT}
 const Variant kTcGridder[] = {
+    TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
+    TGROT2P(32, 16, 4, 2, 4, 2), TGROT2(32, 16, 4, 1, 4), TGROT2P(32, 16, 4, 1, 4, 2), TGROT2P(32, 32, 2, 1, 4, 2), TGROT2(32, 32, 2, 1, 4), TGROT2(32, 16, 4, 2, 4), TGROT2(32, 16, 4, 2, 2), TGROT2(32, 16, 4, 2, 1),
+    TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TGROT(24, 12, 3, 2, 4), TGROT(24, 12, 3, 2, 2), TGROT(24, 12, 3, 1, 2), TGROT(24, 12, 3, 1, 4),
     TGROT(32, 16, 4, 2, 4), TGROT(32, 16, 4, 1, 4), TGROT(32, 16, 4, 1, 2), TGROT(32, 8, 8, 1, 4), TGROT(32, 16, 4, 1, 8),
     TGROT(16, 8, 2, 2, 2), TGROT(16, 8, 2, 2, 4), TGROT(24, 12, 3, 1, 8),
@@ -1071,6 +1345,8 @@ const Variant kTcGridder[] = {
 #undef TGB
 #undef TGR
 #undef TGROT
+#undef TGROT2
+#undef TGROT2P
 #undef TG
 template <int NS, int WARPS, int MINB, int UNR>
 cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
@@ -1088,15 +1364,18 @@ cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
     {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>}
 #define TD(NS, W, MT, MB) \
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>}
+#define TDP(NS, W, MT, MB, P) \
+    {NS, 0, kTensor, 0, "degridder_tcp<" #NS ",W" #W ",MT" #MT ",minB" #MB ",P" #P ">", launch_degridder_tc<NS, W, MT, MB, P>}
 const Variant kTcDegridder[] = {
     TDROT(32, 16, 1, 2), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
     TDROT(24, 8, 4, 1), TDROT(24, 8, 3, 1), TDROT(24, 8, 3, 2), TDROT(16, 8, 4, 1),
     TD(24, 8, 2, 4), TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
-    TD(24, 4, 2, 6),
+    TD(24, 4, 2, 6), TDP(24, 8, 2, 4, 1),
     TD(32, 8, 4, 2), TD(32, 4, 4, 3), TD(32, 8, 8, 1), TD(32, 16, 2, 1),
     TD(16, 8, 4, 2), TD(16, 4, 4, 4), TD(16, 8, 2, 3),
 };
 #undef TD
+#undef TDP
 #undef TDROT
 
 }  // namespace
