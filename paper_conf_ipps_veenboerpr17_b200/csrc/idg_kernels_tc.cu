@@ -1119,6 +1119,121 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 }
 
 // ------------------------------------------------------------------------------------------------
+// degridder_tc2: degridder_tc with the k-block loop split into subgrid rows y and the N~/8 k-blocks of a
+// row (unrolled).  A k-block is 8 pixels of one row, so m is constant over the row: the phase of a
+// (visibility, pixel) slot pair is  u l + (v m_y) + w n  with v m_y formed once per row and visibility,
+// the thread's l pairs (6 distinct values for N~ = 24) kept in registers, and only n read from shared
+// memory per k-block: 2 FFMA2 per row and k-block instead of 3, one LDS instead of two, and the loop
+// overhead spread over a row.
+// ------------------------------------------------------------------------------------------------
+template <int NS, int WARPS, int MT, int MINB>
+__global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc2_kernel(const KernelArgs a) {
+    constexpr int NPIX = NS * NS;
+    constexpr int NXB = NS / 8;   // k-blocks per subgrid row
+    constexpr int h = NS / 2;
+    static_assert(NS % 8 == 0, "k-blocks within a row");
+    extern __shared__ __align__(16) unsigned char smem[];
+    const DegridSmem<NS> sm(smem, a.max_timesteps_in_item);
+    const uint4 *frag_s = sm.frag_s;
+    const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
+    const float *df_s = sm.df_s;
+    __shared__ float red_s[WARPS];
+
+    const int item = a.order[blockIdx.x];
+    const ItemSetup s = dev::item_setup(a, item, NS);
+    const idg_metadata &md = s.md;
+    const int nc = s.nc;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
+    const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s);
+
+    f2p lq[NXB];   // l of the thread's slots q, q+4 in each k-block of a row
+#pragma unroll
+    for (int xb = 0; xb < NXB; ++xb)
+        lq[xb] = pk(float(8 * xb + q - h) * a.cell_l, float(8 * xb + q + 4 - h) * a.cell_l);
+
+    const int nvis = md.nr_timesteps * nc;
+    const int ntiles = (nvis + 15) >> 4;
+    const float rnc = __frcp_rn(float(nc));
+    const bool fdiv = nvis < (1 << 22);
+    auto tstep = [&](int v) { return fdiv ? __float2int_rz((float(v) + 0.5f) * rnc) : v / nc; };
+    const int64_t row = int64_t(a.nr_channels) * 4;
+    float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
+                   int64_t(md.channel_begin) * 4;
+    for (int tile0 = warp * MT; tile0 < ntiles; tile0 += WARPS * MT) {
+        float cu[MT][2], cv[MT][2], cw[MT][2];   // per-visibility coefficients of rows g and g+8
+        float acc[MT][4];
+#pragma unroll
+        for (int i = 0; i < MT; ++i) {
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const int v = (tile0 + i) * 16 + g + 8 * r;
+                float fu = 0.0f, fv = 0.0f, fw = 0.0f;
+                if (v < nvis) {
+                    const int t = tstep(v), c = v - t * nc;
+                    const float4 cB = bq_s[2 * t], cQ = bq_s[2 * t + 1];
+                    const float df = df_s[c];
+                    fu = fmaf(df, cQ.x, cB.x);
+                    fv = fmaf(df, cQ.y, cB.y);
+                    fw = fmaf(df, cQ.z, cB.z);
+                }
+                cu[i][r] = fu;
+                cv[i][r] = fv;
+                cw[i][r] = fw;
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
+        }
+#pragma unroll 1
+        for (int y = 0; y < NS; ++y) {
+            const float m = float(y - h) * a.cell_l;
+            f2p vm[MT][2];
+#pragma unroll
+            for (int i = 0; i < MT; ++i)
+#pragma unroll
+                for (int r = 0; r < 2; ++r) vm[i][r] = dup(cv[i][r] * m);
+#pragma unroll
+            for (int xb = 0; xb < NXB; ++xb) {
+                const int kb = y * NXB + xb;
+                const uint4 bf = frag_s[kb * 32 + lane];
+                const float4 *rec = lmn_s + (kb * 4 + q) * 2 + 1;
+                const float2 nn = *reinterpret_cast<const float2 *>(rec);
+                const f2p n2 = pk(nn.x, nn.y);
+                uint32_t ah[MT][4], al[MT][4];
+#pragma unroll
+                for (int i = 0; i < MT; ++i) {
+                    const float2 p0 = unpk(fma2(dup(cu[i][0]), lq[xb], fma2(dup(cw[i][0]), n2, vm[i][0])));
+                    const float2 p1 = unpk(fma2(dup(cu[i][1]), lq[xb], fma2(dup(cw[i][1]), n2, vm[i][1])));
+                    float sn[4], cs[4];
+                    __sincosf(p0.x, &sn[0], &cs[0]);  // row g,   slot q
+                    __sincosf(p1.x, &sn[1], &cs[1]);  // row g+8, slot q
+                    __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
+                    __sincosf(p1.y, &sn[3], &cs[3]);  // row g+8, slot q+4
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[i][j], al[i][j]);
+                }
+#pragma unroll
+                for (int i = 0; i < MT; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
+#pragma unroll
+                for (int i = 0; i < MT; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
+#pragma unroll
+                for (int i = 0; i < MT; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < MT; ++i) {
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const int v = (tile0 + i) * 16 + g + 8 * r;
+                if (v < nvis) {
+                    const int t = tstep(v), c = v - t * nc;
+                    vis0[int64_t(t) * row + c * 4 + q] = make_float2(acc[i][2 * r] * inv, acc[i][2 * r + 1] * inv);
+                }
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------------------------------------------------
 // Tensor-core degridder with phasor rotation across channel groups (uniform channels, C~ % 32 == 0).
 // A warp takes 32 channels of one timestep as two m-tiles, so each thread's four A rows are the
 // channels c0 + g + 8r (r = 0..3) of the same timestep.  With the phase linear in frequency,
@@ -1127,7 +1242,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 // 1..3 by complex products (fp32, on the FMA pipe) before the operand split.  Exact in exact
 // arithmetic; the rounding is that of up to three extra complex products per phasor.
 // ------------------------------------------------------------------------------------------------
-template <int NS, int WARPS, int MINB, int UNR>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int NKB = NPIX / 8;
@@ -1145,17 +1260,32 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
     const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s);
 
-    const int blocks = nc >> 5;                       // 32-channel blocks per timestep
-    const int nblk = md.nr_timesteps * blocks;
-    const float estep = 8.0f * a.channel_step;
+    // A warp unit is 32 visibilities = 4 channel rows (stride S) for each of the 8 lane groups g:
+    //   CPT = 0 (C~ % 32 == 0): one timestep, 32-channel block, lane base channel g, S = 8;
+    //   CPT = 4, 8, 16 (every item exactly CPT channels): 32 / CPT timesteps per unit, CPT / 4 lane groups
+    //   per timestep, lane base channel g % (CPT / 4), S = CPT / 4.
+    static_assert(CPT == 0 || CPT == 4 || CPT == 8 || CPT == 16, "channels per timestep");
+    constexpr int S = CPT ? CPT / 4 : 8;
+    const int blocks = CPT ? 1 : nc >> 5;              // units per timestep (CPT = 0)
+    const int nblk = CPT ? (md.nr_timesteps * CPT + 31) / 32 : md.nr_timesteps * blocks;
+    const float estep = float(S) * a.channel_step;
     const int64_t row = int64_t(a.nr_channels) * 4;
     float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
                    int64_t(md.channel_begin) * 4;
     for (int bk = warp; bk < nblk; bk += WARPS) {
-        const int t = bk / blocks, c0 = (bk - t * blocks) * 32;
-        const float4 cB = bq_s[2 * t], cQ = bq_s[2 * t + 1];
-        const float df = df_s[c0 + g];
-        // row 0 (channel c0 + g) coefficients, and the coefficients of the E phase
+        int t, c0;
+        if constexpr (CPT) {
+            t = bk * (32 / CPT) + g / S;
+            c0 = g % S;
+        } else {
+            t = bk / blocks;
+            c0 = (bk - t * blocks) * 32 + g;
+        }
+        const bool valid = t < md.nr_timesteps;
+        const int tc = valid ? t : md.nr_timesteps - 1;
+        const float4 cB = bq_s[2 * tc], cQ = bq_s[2 * tc + 1];
+        const float df = df_s[c0];
+        // row 0 (channel c0) coefficients, and the coefficients of the E phase
         const f2p cu = dup(fmaf(df, cQ.x, cB.x)), cv = dup(fmaf(df, cQ.y, cB.y)), cw = dup(fmaf(df, cQ.z, cB.z));
         const f2p eu = dup(estep * cQ.x), ev = dup(estep * cQ.y), ew = dup(estep * cQ.z);
         float acc[2][4];
@@ -1199,10 +1329,12 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
 #pragma unroll
             for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
         }
-        float2 *vt = vis0 + int64_t(t) * row + int64_t(c0 + g) * 4 + q;
+        if (valid) {
+            float2 *vt = vis0 + int64_t(t) * row + int64_t(c0) * 4 + q;
 #pragma unroll
-        for (int r = 0; r < 4; ++r)
-            vt[r * 32] = make_float2(acc[r >> 1][2 * (r & 1)] * inv, acc[r >> 1][2 * (r & 1) + 1] * inv);
+            for (int r = 0; r < 4; ++r)
+                vt[r * S * 4] = make_float2(acc[r >> 1][2 * (r & 1)] * inv, acc[r >> 1][2 * (r & 1) + 1] * inv);
+        }
     }
 }
 
@@ -1348,27 +1480,48 @@ const Variant kTcGridder[] = {
 #undef TGROT2
 #undef TGROT2P
 #undef TG
-template <int NS, int WARPS, int MINB, int UNR>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0>
 cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
     cudaError_t terr = ensure_dft_tables();
     if (terr != cudaSuccess) return terr;
     const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
-    cudaError_t err = dev::prepare(degridder_rot_kernel<NS, WARPS, MINB, UNR>, smem);
+    cudaError_t err = dev::prepare(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("degridder", st);
-    degridder_rot_kernel<NS, WARPS, MINB, UNR><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 
+// every item exactly CPT (4, 8 or 16) channels
+#define TDROTC(NS, W, MB, U, CPT) \
+    {NS, CPT, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT>, CPT}
 #define TDROT(NS, W, MB, U) \
     {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>}
 #define TD(NS, W, MT, MB) \
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>}
+template <int NS, int WARPS, int MT, int MINB>
+cudaError_t launch_degridder_tc2(const KernelArgs &a, cudaStream_t st) {
+    cudaError_t terr = ensure_dft_tables();
+    if (terr != cudaSuccess) return terr;
+    const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
+    cudaError_t err = dev::prepare(degridder_tc2_kernel<NS, WARPS, MT, MINB>, smem);
+    if (err != cudaSuccess) return err;
+    LaunchScope scope("degridder", st);
+    degridder_tc2_kernel<NS, WARPS, MT, MINB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    return cudaGetLastError();
+}
+#define TD2(NS, W, MT, MB) \
+    {NS, 0, kTensor, 0, "degridder_tc2<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc2<NS, W, MT, MB>}
 #define TDP(NS, W, MT, MB, P) \
     {NS, 0, kTensor, 0, "degridder_tcp<" #NS ",W" #W ",MT" #MT ",minB" #MB ",P" #P ">", launch_degridder_tc<NS, W, MT, MB, P>}
 const Variant kTcDegridder[] = {
     TDROT(32, 16, 1, 2), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
     TDROT(24, 8, 4, 1), TDROT(24, 8, 3, 1), TDROT(24, 8, 3, 2), TDROT(16, 8, 4, 1),
+    TDROTC(24, 8, 4, 1, 16), TDROTC(24, 8, 3, 1, 16), TDROTC(24, 8, 4, 1, 8), TDROTC(24, 8, 4, 1, 4),
+    TDROTC(32, 16, 1, 2, 16), TDROTC(32, 16, 1, 2, 8), TDROTC(32, 16, 1, 2, 4),
+    TDROTC(16, 8, 4, 1, 16), TDROTC(16, 8, 4, 1, 8), TDROTC(16, 8, 4, 1, 4),
+    TD2(24, 8, 2, 4), TD2(24, 8, 2, 3), TD2(24, 8, 4, 2), TD2(32, 8, 2, 4), TD2(16, 8, 2, 4),
     TD(24, 8, 2, 4), TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
     TD(24, 4, 2, 6), TDP(24, 8, 2, 4, 1),
     TD(32, 8, 4, 2), TD(32, 4, 4, 3), TD(32, 8, 8, 1), TD(32, 16, 2, 1),
@@ -1376,7 +1529,9 @@ const Variant kTcDegridder[] = {
 };
 #undef TD
 #undef TDP
+#undef TD2
 #undef TDROT
+#undef TDROTC
 
 }  // namespace
 
