@@ -1454,11 +1454,15 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 #define TGROT2(NS, W, MT, MB, KPT) \
     {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ">", \
      launch_gridder_rot2<NS, W, MT, MB, KPT, KPT, 128>, 8 * KPT}
+#define TGROT2K(NS, W, MT, MB, KPT, KB) \
+    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",KB" #KB ">", \
+     launch_gridder_rot2<NS, W, MT, MB, KPT, KPT, KB>, 8 * KPT}
 #define TGROT2P(NS, W, MT, MB, KPT, GP) \
     {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP ">", \
      launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128>, 8 * KPT}
 const Variant kTcGridder[] = {
     TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
+    TGROT2K(24, 12, 3, 2, 2, 64),
     TGROT2P(32, 16, 4, 2, 4, 2), TGROT2(32, 16, 4, 1, 4), TGROT2P(32, 16, 4, 1, 4, 2), TGROT2P(32, 32, 2, 1, 4, 2), TGROT2(32, 32, 2, 1, 4), TGROT2(32, 16, 4, 2, 4), TGROT2(32, 16, 4, 2, 2), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TGROT(24, 12, 3, 2, 4), TGROT(24, 12, 3, 2, 2), TGROT(24, 12, 3, 1, 2), TGROT(24, 12, 3, 1, 4),
@@ -1479,6 +1483,7 @@ const Variant kTcGridder[] = {
 #undef TGROT
 #undef TGROT2
 #undef TGROT2P
+#undef TGROT2K
 #undef TG
 template <int NS, int WARPS, int MINB, int UNR, int CPT = 0>
 cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
@@ -1516,10 +1521,10 @@ cudaError_t launch_degridder_tc2(const KernelArgs &a, cudaStream_t st) {
 #define TDP(NS, W, MT, MB, P) \
     {NS, 0, kTensor, 0, "degridder_tcp<" #NS ",W" #W ",MT" #MT ",minB" #MB ",P" #P ">", launch_degridder_tc<NS, W, MT, MB, P>}
 const Variant kTcDegridder[] = {
-    TDROT(32, 16, 1, 2), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
+    TDROT(32, 16, 1, 2), TDROT(32, 16, 2, 1), TDROT(32, 16, 2, 2), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
     TDROT(24, 8, 4, 1), TDROT(24, 8, 3, 1), TDROT(24, 8, 3, 2), TDROT(16, 8, 4, 1),
-    TDROTC(24, 8, 4, 1, 16), TDROTC(24, 8, 3, 1, 16), TDROTC(24, 8, 4, 1, 8), TDROTC(24, 8, 4, 1, 4),
-    TDROTC(32, 16, 1, 2, 16), TDROTC(32, 16, 1, 2, 8), TDROTC(32, 16, 1, 2, 4),
+    TDROTC(24, 8, 4, 1, 16), TDROTC(24, 8, 3, 1, 16), TDROTC(24, 16, 2, 1, 16), TDROTC(24, 8, 4, 1, 8), TDROTC(24, 8, 4, 1, 4),
+    TDROTC(32, 16, 1, 2, 16), TDROTC(32, 16, 2, 1, 16), TDROTC(32, 16, 2, 2, 16), TDROTC(32, 16, 1, 2, 8), TDROTC(32, 16, 1, 2, 4),
     TDROTC(16, 8, 4, 1, 16), TDROTC(16, 8, 4, 1, 8), TDROTC(16, 8, 4, 1, 4),
     TD2(24, 8, 2, 4), TD2(24, 8, 2, 3), TD2(24, 8, 4, 2), TD2(32, 8, 2, 4), TD2(16, 8, 2, 4),
     TD(24, 8, 2, 4), TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
