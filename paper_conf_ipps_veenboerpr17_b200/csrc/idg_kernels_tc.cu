@@ -1463,7 +1463,7 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 const Variant kTcGridder[] = {
     TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
     TGROT2K(24, 12, 3, 2, 2, 64),
-    TGROT2P(32, 16, 4, 2, 4, 2), TGROT2(32, 16, 4, 1, 4), TGROT2P(32, 16, 4, 1, 4, 2), TGROT2P(32, 32, 2, 1, 4, 2), TGROT2(32, 32, 2, 1, 4), TGROT2(32, 16, 4, 2, 4), TGROT2(32, 16, 4, 2, 2), TGROT2(32, 16, 4, 2, 1),
+    TGROT2P(32, 16, 4, 2, 4, 2), TGROT2(32, 16, 4, 1, 4), TGROT2P(32, 16, 4, 1, 4, 2), TGROT2P(32, 32, 2, 1, 4, 2), TGROT2(32, 32, 2, 1, 4), TGROT2(32, 16, 4, 2, 4), TGROT2(32, 16, 4, 2, 2), TGROT2(32, 16, 4, 1, 2), TGROT2(32, 32, 2, 1, 2), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TGROT(24, 12, 3, 2, 4), TGROT(24, 12, 3, 2, 2), TGROT(24, 12, 3, 1, 2), TGROT(24, 12, 3, 1, 4),
     TGROT(32, 16, 4, 2, 4), TGROT(32, 16, 4, 1, 4), TGROT(32, 16, 4, 1, 2), TGROT(32, 8, 8, 1, 4), TGROT(32, 16, 4, 1, 8),
@@ -1521,10 +1521,10 @@ cudaError_t launch_degridder_tc2(const KernelArgs &a, cudaStream_t st) {
 #define TDP(NS, W, MT, MB, P) \
     {NS, 0, kTensor, 0, "degridder_tcp<" #NS ",W" #W ",MT" #MT ",minB" #MB ",P" #P ">", launch_degridder_tc<NS, W, MT, MB, P>}
 const Variant kTcDegridder[] = {
-    TDROT(32, 16, 1, 2), TDROT(32, 16, 2, 1), TDROT(32, 16, 2, 2), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
+    TDROT(32, 16, 2, 2), TDROT(32, 16, 1, 2), TDROT(32, 16, 2, 1), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
     TDROT(24, 8, 4, 1), TDROT(24, 8, 3, 1), TDROT(24, 8, 3, 2), TDROT(16, 8, 4, 1),
     TDROTC(24, 8, 4, 1, 16), TDROTC(24, 8, 3, 1, 16), TDROTC(24, 16, 2, 1, 16), TDROTC(24, 8, 4, 1, 8), TDROTC(24, 8, 4, 1, 4),
-    TDROTC(32, 16, 1, 2, 16), TDROTC(32, 16, 2, 1, 16), TDROTC(32, 16, 2, 2, 16), TDROTC(32, 16, 1, 2, 8), TDROTC(32, 16, 1, 2, 4),
+    TDROTC(32, 16, 2, 1, 16), TDROTC(32, 16, 1, 2, 16), TDROTC(32, 16, 2, 2, 16), TDROTC(32, 16, 2, 1, 8), TDROTC(32, 16, 2, 1, 4),
     TDROTC(16, 8, 4, 1, 16), TDROTC(16, 8, 4, 1, 8), TDROTC(16, 8, 4, 1, 4),
     TD2(24, 8, 2, 4), TD2(24, 8, 2, 3), TD2(24, 8, 4, 2), TD2(32, 8, 2, 4), TD2(16, 8, 2, 4),
     TD(24, 8, 2, 4), TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
