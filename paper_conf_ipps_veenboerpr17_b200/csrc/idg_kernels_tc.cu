@@ -1242,7 +1242,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc2_kernel(const K
 // 1..3 by complex products (fp32, on the FMA pipe) before the operand split.  Exact in exact
 // arithmetic; the rounding is that of up to three extra complex products per phasor.
 // ------------------------------------------------------------------------------------------------
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int NKB = NPIX / 8;
@@ -1260,23 +1260,26 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
     const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s);
 
-    // A warp unit is 32 visibilities = 4 channel rows (stride S) for each of the 8 lane groups g:
-    //   CPT = 0 (C~ % 32 == 0): one timestep, 32-channel block, lane base channel g, S = 8;
-    //   CPT = 4, 8, 16 (every item exactly CPT channels): 32 / CPT timesteps per unit, CPT / 4 lane groups
-    //   per timestep, lane base channel g % (CPT / 4), S = CPT / 4.
-    static_assert(CPT == 0 || CPT == 4 || CPT == 8 || CPT == 16, "channels per timestep");
-    constexpr int S = CPT ? CPT / 4 : 8;
+    // A warp unit is 8 R visibilities = R channel rows (stride CS) for each of the 8 lane groups g, as R / 2
+    // m-tiles (lane group g owns rows g and g+8 of every tile):
+    //   CPT = 0 (C~ % 32 == 0, R = 4): one timestep, 32-channel block, lane base channel g, CS = 8;
+    //   CPT > 0 (every item exactly CPT channels): CPT / R lane groups per timestep, 8 R / CPT timesteps per
+    //   unit, lane base channel g % (CPT / R), CS = CPT / R.
+    static_assert(R == 4 || R == 8 || R == 16, "channel rows per lane");
+    static_assert(CPT == 0 ? R == 4 : (CPT % R == 0 && (8 * R) % CPT == 0), "channels per timestep");
+    constexpr int NTL = R / 2;                        // m-tiles per unit
+    constexpr int CS = CPT ? CPT / R : 8;             // channel stride of a lane's rows
     const int blocks = CPT ? 1 : nc >> 5;              // units per timestep (CPT = 0)
-    const int nblk = CPT ? (md.nr_timesteps * CPT + 31) / 32 : md.nr_timesteps * blocks;
-    const float estep = float(S) * a.channel_step;
+    const int nblk = CPT ? (md.nr_timesteps * CPT + 8 * R - 1) / (8 * R) : md.nr_timesteps * blocks;
+    const float estep = float(CS) * a.channel_step;
     const int64_t row = int64_t(a.nr_channels) * 4;
     float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
                    int64_t(md.channel_begin) * 4;
     for (int bk = warp; bk < nblk; bk += WARPS) {
         int t, c0;
         if constexpr (CPT) {
-            t = bk * (32 / CPT) + g / S;
-            c0 = g % S;
+            t = bk * (8 * R / CPT) + g / CS;
+            c0 = g % CS;
         } else {
             t = bk / blocks;
             c0 = (bk - t * blocks) * 32 + g;
@@ -1288,9 +1291,9 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
         // row 0 (channel c0) coefficients, and the coefficients of the E phase
         const f2p cu = dup(fmaf(df, cQ.x, cB.x)), cv = dup(fmaf(df, cQ.y, cB.y)), cw = dup(fmaf(df, cQ.z, cB.z));
         const f2p eu = dup(estep * cQ.x), ev = dup(estep * cQ.y), ew = dup(estep * cQ.z);
-        float acc[2][4];
+        float acc[NTL][4];
 #pragma unroll
-        for (int i = 0; i < 2; ++i)
+        for (int i = 0; i < NTL; ++i)
 #pragma unroll
             for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
         static_assert(NKB % UNR == 0, "k-block unroll");
@@ -1306,34 +1309,54 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
             __sincosf(p.y, &s1, &c1q);
             __sincosf(e.x, &es0, &ec0);
             __sincosf(e.y, &es1, &ec1);
-            // rows r = 0..3 at slots (q, q+4), packed: C = (cos, cos), S = (sin, sin)
+            // rows r = 0..R-1 at slots (q, q+4), packed: C = (cos, cos), S = (sin, sin)
             f2p C = pk(c0q, c1q), S = pk(s0, s1);
             const f2p EC = pk(ec0, ec1), ES = pk(es0, es1), NES = pk(-es0, -es1);
-            uint32_t ah[2][4], al[2][4];
+            if constexpr (R == 4) {
+                uint32_t ah[2][4], al[2][4];
 #pragma unroll
-            for (int r = 0; r < 4; ++r) {
-                if (r > 0) {
-                    const f2p Cn = fma2(C, EC, mul2(S, NES));
-                    S = fma2(C, ES, mul2(S, EC));
-                    C = Cn;
+                for (int r = 0; r < 4; ++r) {
+                    if (r > 0) {
+                        const f2p Cn = fma2(C, EC, mul2(S, NES));
+                        S = fma2(C, ES, mul2(S, EC));
+                        C = Cn;
+                    }
+                    const float2 cc = unpk(C), ss = unpk(S);
+                    // tile r >> 1, row g (r even) / g+8 (r odd): A regs {(row, q), (row+8, q), (row, q+4), (row+8, q+4)}
+                    split_phasor(cc.x, ss.x, ah[r >> 1][r & 1], al[r >> 1][r & 1]);
+                    split_phasor(cc.y, ss.y, ah[r >> 1][2 + (r & 1)], al[r >> 1][2 + (r & 1)]);
                 }
-                const float2 cc = unpk(C), ss = unpk(S);
-                // tile r >> 1, row g (r even) / g+8 (r odd): A regs {(row, q), (row+8, q), (row, q+4), (row+8, q+4)}
-                split_phasor(cc.x, ss.x, ah[r >> 1][r & 1], al[r >> 1][r & 1]);
-                split_phasor(cc.y, ss.y, ah[r >> 1][2 + (r & 1)], al[r >> 1][2 + (r & 1)]);
+#pragma unroll
+                for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
+#pragma unroll
+                for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
+#pragma unroll
+                for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
+            } else {
+                // R = 8, 16: each tile's three products issued as soon as its two rows are split
+#pragma unroll
+                for (int i = 0; i < NTL; ++i) {
+                    uint32_t ah[4], al[4];
+#pragma unroll
+                    for (int h2 = 0; h2 < 2; ++h2) {
+                        if (i > 0 || h2 > 0) {
+                            const f2p Cn = fma2(C, EC, mul2(S, NES));
+                            S = fma2(C, ES, mul2(S, EC));
+                            C = Cn;
+                        }
+                        const float2 cc = unpk(C), ss = unpk(S);
+                        split_phasor(cc.x, ss.x, ah[h2], al[h2]);
+                        split_phasor(cc.y, ss.y, ah[2 + h2], al[2 + h2]);
+                    }
+                    mma3(acc[i], ah, al, bf);
+                }
             }
-#pragma unroll
-            for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
-#pragma unroll
-            for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
-#pragma unroll
-            for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
         }
         if (valid) {
             float2 *vt = vis0 + int64_t(t) * row + int64_t(c0) * 4 + q;
 #pragma unroll
-            for (int r = 0; r < 4; ++r)
-                vt[r * S * 4] = make_float2(acc[r >> 1][2 * (r & 1)] * inv, acc[r >> 1][2 * (r & 1) + 1] * inv);
+            for (int r = 0; r < R; ++r)
+                vt[r * CS * 4] = make_float2(acc[r >> 1][2 * (r & 1)] * inv, acc[r >> 1][2 * (r & 1) + 1] * inv);
         }
     }
 }
@@ -1485,15 +1508,15 @@ const Variant kTcGridder[] = {
 #undef TGROT2P
 #undef TGROT2K
 #undef TG
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4>
 cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
     cudaError_t terr = ensure_dft_tables();
     if (terr != cudaSuccess) return terr;
     const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
-    cudaError_t err = dev::prepare(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT>, smem);
+    cudaError_t err = dev::prepare(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("degridder", st);
-    degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -1501,6 +1524,13 @@ cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
 #define TDROTC(NS, W, MB, U, CPT) \
     {NS, CPT, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT>, CPT}
+// R = 8 channel rows per lane (4 m-tiles per unit), every item exactly CPT channels
+#define TDROT8(NS, W, MB, U, CPT) \
+    {NS, CPT, kTensor, 1, "degridder_rot8<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, 8>, CPT}
+#define TDROT16(NS, W, MB, U, CPT) \
+    {NS, CPT, kTensor, 1, "degridder_rot16<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, 16>, CPT}
 #define TDROT(NS, W, MB, U) \
     {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>}
 #define TD(NS, W, MT, MB) \
@@ -1521,6 +1551,8 @@ cudaError_t launch_degridder_tc2(const KernelArgs &a, cudaStream_t st) {
 #define TDP(NS, W, MT, MB, P) \
     {NS, 0, kTensor, 0, "degridder_tcp<" #NS ",W" #W ",MT" #MT ",minB" #MB ",P" #P ">", launch_degridder_tc<NS, W, MT, MB, P>}
 const Variant kTcDegridder[] = {
+    TDROT16(24, 4, 3, 1, 16), TDROT16(24, 8, 2, 1, 16), TDROT8(24, 8, 2, 1, 16), TDROT8(24, 8, 3, 1, 16),
+    TDROT16(32, 8, 2, 1, 32), TDROT16(32, 8, 2, 1, 16), TDROT16(32, 16, 1, 1, 32), TDROT16(16, 8, 2, 1, 16), TDROT16(16, 8, 2, 1, 32), TDROT8(32, 16, 2, 1, 16), TDROT8(32, 16, 2, 1, 32), TDROT8(24, 8, 2, 1, 8), TDROT8(32, 16, 2, 1, 8), TDROT8(16, 8, 2, 1, 8),
     TDROT(32, 16, 2, 2), TDROT(32, 16, 1, 2), TDROT(32, 16, 2, 1), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
     TDROT(24, 8, 4, 1), TDROT(24, 8, 3, 1), TDROT(24, 8, 3, 2), TDROT(16, 8, 4, 1),
     TDROTC(24, 8, 4, 1, 16), TDROTC(24, 8, 3, 1, 16), TDROTC(24, 16, 2, 1, 16), TDROTC(24, 8, 4, 1, 8), TDROTC(24, 8, 4, 1, 4),
@@ -1537,6 +1569,8 @@ const Variant kTcDegridder[] = {
 #undef TD2
 #undef TDROT
 #undef TDROTC
+#undef TDROT8
+#undef TDROT16
 
 }  // namespace
 
