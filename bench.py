@@ -200,7 +200,8 @@ def sincos_per_pair(variant: str, nc_item: int) -> float:
     of the 4 lanes sharing the pixel, for 8 J pairs (J = channel groups of 8); gridder_rot2: the 8 slot
     phasors only (E_t derived from slots q, q+4); gridder_tcr: half the
     phasors by recurrence plus one step phasor per (pixel, timestep) in each of the 2 lanes;
-    degridder_rot: per (visibility row 0, pixel) one phasor and one rotation E for four channel rows."""
+    degridder_rot / rot8 / rot16: per (visibility row 0, pixel) one phasor and one rotation E for 4 / 8 / 16
+    channel rows."""
     j = max(1, nc_item // 8)
     if variant.startswith("gridder_rot2"):
         return 1.0 / j  # the 8 group-0 phasors only; E_t is derived from them (no sincos)
@@ -208,6 +209,10 @@ def sincos_per_pair(variant: str, nc_item: int) -> float:
         return (8.0 + (4.0 if j > 1 else 0.0)) / (8.0 * j)
     if variant.startswith("gridder_tcr"):
         return 0.5 + 0.5 / j
+    if variant.startswith("degridder_rot16"):
+        return 2.0 / 16  # per pixel slot: row 0 and E_tp for 16 channel rows
+    if variant.startswith("degridder_rot8"):
+        return 2.0 / 8
     if variant.startswith("degridder_rot"):
         return 0.5     # per pixel slot: row 0 and E_tp for 4 channel rows
     return 1.0
