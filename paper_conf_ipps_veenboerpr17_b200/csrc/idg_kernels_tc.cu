@@ -80,6 +80,25 @@ __device__ __forceinline__ void split2(float x, float y, uint32_t &hi, uint32_t 
 }
 __device__ __forceinline__ void split_phasor(float x, float y, uint32_t &hi, uint32_t &lo) { split2(x, y, hi, lo); }
 
+// (x, y) -> f16x2 hi = rn(x, y) and the exact fp32 residuals x - hi, y - hi (two FHFMA, no repacking):
+// the residuals feed a tf32 mma directly (it reads the top 19 bits of each fp32 register).
+__device__ __forceinline__ void split_hi_res(float x, float y, uint32_t &hi, float &dx, float &dy) {
+    hi = h2_bits(__floats2half2_rn(x, y));
+    asm("{\n.reg .f16 a, b, m;\nmov.b32 {a, b}, %2;\nmov.b16 m, 0xBC00;\n"
+        "fma.rn.f32.f16 %0, a, m, %3;\nfma.rn.f32.f16 %1, b, m, %4;\n}"
+        : "=f"(dx), "=f"(dy) : "r"(hi), "f"(x), "f"(y));
+}
+
+// D += A B, m16n8k8 tf32 (fp32 registers; A {(g, q), (g+8, q), (g, q+4), (g+8, q+4)}, B {(q, g), (q+4, g)}).
+__device__ __forceinline__ void mma1688_tf32(float (&d)[4], float a0, float a1, float a2, float a3, float b0,
+                                             float b1) {
+    asm("mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(__float_as_uint(a0)), "r"(__float_as_uint(a1)), "r"(__float_as_uint(a2)), "r"(__float_as_uint(a3)),
+          "r"(__float_as_uint(b0)), "r"(__float_as_uint(b1)));
+}
+
 __device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
                                          uint32_t b0, uint32_t b1) {
     asm("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
@@ -1242,7 +1261,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc2_kernel(const K
 // 1..3 by complex products (fp32, on the FMA pipe) before the operand split.  Exact in exact
 // arithmetic; the rounding is that of up to three extra complex products per phasor.
 // ------------------------------------------------------------------------------------------------
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int TFL = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int NKB = NPIX / 8;
@@ -1334,21 +1353,49 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                 for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
             } else {
                 // R = 8, 16: each tile's three products issued as soon as its two rows are split
+                if constexpr (TFL) {
+                    // lo(A) B_hi as two tf32 m16n8k8 (slots q and q+4) on the fp32 residuals: no lo repacking.
+                    // B_hi as fp32: the lane's f16 pairs {B[2q][g], B[2q+1][g]} (cos / sin rows of slot q)
+                    // are exactly the tf32 B registers {(k = q, g), (k = q+4, g)} of the slot-q product.
+                    const float2 b0 = __half22float2(*reinterpret_cast<const __half2 *>(&bf.x));
+                    const float2 b4 = __half22float2(*reinterpret_cast<const __half2 *>(&bf.y));
 #pragma unroll
-                for (int i = 0; i < NTL; ++i) {
-                    uint32_t ah[4], al[4];
+                    for (int i = 0; i < NTL; ++i) {
+                        uint32_t ah[4];
+                        float lc[4], ls[4];
 #pragma unroll
-                    for (int h2 = 0; h2 < 2; ++h2) {
-                        if (i > 0 || h2 > 0) {
-                            const f2p Cn = fma2(C, EC, mul2(S, NES));
-                            S = fma2(C, ES, mul2(S, EC));
-                            C = Cn;
+                        for (int h2 = 0; h2 < 2; ++h2) {
+                            if (i > 0 || h2 > 0) {
+                                const f2p Cn = fma2(C, EC, mul2(S, NES));
+                                S = fma2(C, ES, mul2(S, EC));
+                                C = Cn;
+                            }
+                            const float2 cc = unpk(C), ss = unpk(S);
+                            split_hi_res(cc.x, ss.x, ah[h2], lc[h2], ls[h2]);
+                            split_hi_res(cc.y, ss.y, ah[2 + h2], lc[2 + h2], ls[2 + h2]);
                         }
-                        const float2 cc = unpk(C), ss = unpk(S);
-                        split_phasor(cc.x, ss.x, ah[h2], al[h2]);
-                        split_phasor(cc.y, ss.y, ah[2 + h2], al[2 + h2]);
+                        mma16816(acc[i], ah[0], ah[1], ah[2], ah[3], bf.x, bf.y);
+                        mma16816(acc[i], ah[0], ah[1], ah[2], ah[3], bf.z, bf.w);
+                        mma1688_tf32(acc[i], lc[0], lc[1], ls[0], ls[1], b0.x, b0.y);
+                        mma1688_tf32(acc[i], lc[2], lc[3], ls[2], ls[3], b4.x, b4.y);
                     }
-                    mma3(acc[i], ah, al, bf);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < NTL; ++i) {
+                        uint32_t ah[4], al[4];
+#pragma unroll
+                        for (int h2 = 0; h2 < 2; ++h2) {
+                            if (i > 0 || h2 > 0) {
+                                const f2p Cn = fma2(C, EC, mul2(S, NES));
+                                S = fma2(C, ES, mul2(S, EC));
+                                C = Cn;
+                            }
+                            const float2 cc = unpk(C), ss = unpk(S);
+                            split_phasor(cc.x, ss.x, ah[h2], al[h2]);
+                            split_phasor(cc.y, ss.y, ah[2 + h2], al[2 + h2]);
+                        }
+                        mma3(acc[i], ah, al, bf);
+                    }
                 }
             }
         }
@@ -1508,15 +1555,15 @@ const Variant kTcGridder[] = {
 #undef TGROT2P
 #undef TGROT2K
 #undef TG
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int TFL = 0>
 cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
     cudaError_t terr = ensure_dft_tables();
     if (terr != cudaSuccess) return terr;
     const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
-    cudaError_t err = dev::prepare(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R>, smem);
+    cudaError_t err = dev::prepare(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R, TFL>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("degridder", st);
-    degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R, TFL><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -1531,6 +1578,10 @@ cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
 #define TDROT16(NS, W, MB, U, CPT) \
     {NS, CPT, kTensor, 1, "degridder_rot16<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, 16>, CPT}
+// R = 16 with the lo(A) B_hi product as tf32 mma on the fp32 residuals
+#define TDROT16T(NS, W, MB, U, CPT) \
+    {NS, CPT, kTensor, 1, "degridder_rot16t<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, 16, 1>, CPT}
 #define TDROT(NS, W, MB, U) \
     {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>}
 #define TD(NS, W, MT, MB) \
@@ -1560,7 +1611,7 @@ const Variant kTcDegridder[] = {
     TDROTC(16, 8, 4, 1, 16), TDROTC(16, 8, 4, 1, 8), TDROTC(16, 8, 4, 1, 4),
     TD2(24, 8, 2, 4), TD2(24, 8, 2, 3), TD2(24, 8, 4, 2), TD2(32, 8, 2, 4), TD2(16, 8, 2, 4),
     TD(24, 8, 2, 4), TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
-    TD(24, 4, 2, 6), TDP(24, 8, 2, 4, 1),
+    TD(24, 4, 2, 6), TDP(24, 8, 2, 4, 1), TDROT16T(24, 4, 3, 1, 16),
     TD(32, 8, 4, 2), TD(32, 4, 4, 3), TD(32, 8, 8, 1), TD(32, 16, 2, 1),
     TD(16, 8, 4, 2), TD(16, 4, 4, 4), TD(16, 8, 2, 3),
 };
@@ -1571,6 +1622,7 @@ const Variant kTcDegridder[] = {
 #undef TDROTC
 #undef TDROT8
 #undef TDROT16
+#undef TDROT16T
 
 }  // namespace
 

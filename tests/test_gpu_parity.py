@@ -80,6 +80,7 @@ KINDS = {
     "rot2": ("gridder_rot2<*", "degridder_rot<*"), # rotation with E_t derived from the slot phasors
     "rot8": ("gridder_rot2<*", "degridder_rot8<*"), # degridder: 8 channel rows per lane (0.25 sincos/pair)
     "rot16": ("gridder_rot2<*", "degridder_rot16<*"), # degridder: 16 channel rows per lane
+    "rot16t": ("gridder_rot2<*", "degridder_rot16t<*"), # + lo(A) B_hi as tf32 mma
     "tc2": ("gridder_rot2<*", "degridder_tc2<*"), # degridder: row-split phase (m per row, l in registers)
     "poly": ("gridder_rot2<*", "degridder_tcp<*"), # degridder with part of the sincos on the FMA pipe
     "tf32": ("gridder_tf32*", "degridder_tf32*"),  # split-tf32 tensor-core kernels
