@@ -710,7 +710,7 @@ __device__ __forceinline__ f2p add2(f2p a, f2p b) {
     return r;
 }
 
-template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB>
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB, int TU = 1>
 __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const KernelArgs a) {
     constexpr int NT = WARPS * 32;
     constexpr int NPIX = NS * NS;
@@ -810,7 +810,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
         }
         __syncthreads();
         // (5) per timestep: group-0 phasors of every tile, E_t from them, one fresh D_j per group j > 0
-#pragma unroll 1
+#pragma unroll TU
         for (int t = t0; t < t1; ++t) {
             const float4 cB = coef_s[2 * (t - t0)], cQ = coef_s[2 * (t - t0) + 1];
             // slot coefficients c_s = B_t + df_s Q_t (u, v, w components)
@@ -1483,15 +1483,15 @@ cudaError_t launch_gridder_rot(const KernelArgs &a, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB>
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int TU = 1>
 cudaError_t launch_gridder_rot2(const KernelArgs &a, cudaStream_t st) {
     cudaError_t terr = ensure_dft_tables();
     if (terr != cudaSuccess) return terr;
     const size_t smem = gridder_rot_smem_bytes(NS, KBB);
-    cudaError_t err = dev::prepare(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB>, smem);
+    cudaError_t err = dev::prepare(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, TU>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("gridder", st);
-    gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, TU><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -1602,8 +1602,8 @@ cudaError_t launch_degridder_tc2(const KernelArgs &a, cudaStream_t st) {
 #define TDP(NS, W, MT, MB, P) \
     {NS, 0, kTensor, 0, "degridder_tcp<" #NS ",W" #W ",MT" #MT ",minB" #MB ",P" #P ">", launch_degridder_tc<NS, W, MT, MB, P>}
 const Variant kTcDegridder[] = {
-    TDROT16(24, 4, 3, 1, 16), TDROT16(24, 8, 2, 1, 16), TDROT8(24, 8, 2, 1, 16), TDROT8(24, 8, 3, 1, 16),
-    TDROT16(32, 8, 2, 1, 32), TDROT16(32, 8, 2, 1, 16), TDROT16(32, 16, 1, 1, 32), TDROT16(16, 8, 2, 1, 16), TDROT16(16, 8, 2, 1, 32), TDROT8(32, 16, 2, 1, 16), TDROT8(32, 16, 2, 1, 32), TDROT8(24, 8, 2, 1, 8), TDROT8(32, 16, 2, 1, 8), TDROT8(16, 8, 2, 1, 8),
+    TDROT16(24, 4, 3, 4, 16), TDROT16(24, 4, 3, 2, 16), TDROT16(24, 4, 3, 1, 16), TDROT16(24, 8, 2, 1, 16), TDROT8(24, 8, 2, 1, 16), TDROT8(24, 8, 3, 1, 16),
+    TDROT16(32, 8, 2, 2, 32), TDROT16(32, 8, 2, 2, 16), TDROT16(32, 8, 2, 1, 32), TDROT16(32, 8, 2, 1, 16), TDROT16(32, 16, 1, 1, 32), TDROT16(16, 8, 2, 1, 16), TDROT16(16, 8, 2, 1, 32), TDROT8(32, 16, 2, 1, 16), TDROT8(32, 16, 2, 1, 32), TDROT8(24, 8, 2, 1, 8), TDROT8(32, 16, 2, 1, 8), TDROT8(16, 8, 2, 1, 8),
     TDROT(32, 16, 2, 2), TDROT(32, 16, 1, 2), TDROT(32, 16, 2, 1), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
     TDROT(24, 8, 4, 1), TDROT(24, 8, 3, 1), TDROT(24, 8, 3, 2), TDROT(16, 8, 4, 1),
     TDROTC(24, 8, 4, 1, 16), TDROTC(24, 8, 3, 1, 16), TDROTC(24, 16, 2, 1, 16), TDROTC(24, 8, 4, 1, 8), TDROTC(24, 8, 4, 1, 4),
