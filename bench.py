@@ -432,21 +432,31 @@ def run_ours(args):
             traffic = json.load(open(prof_json)).get(args.config, {}).get(dominant, {}).get("dram_bytes")
         except Exception:
             traffic = None
+    # peak: the one-sincos-per-pair roofline from the unit counts at the clock of the timed region
+    # (148 SMs x 16 MUFU lanes/clk / 2 MUFU per sincos x 36 paper-ops per pair).  It is a hard ceiling for
+    # the paper's formulation (one sincos per pair); the rotation kernels evaluate fewer
+    # sincos, so for them it is the paper-metric ceiling, and their own sincos bound is reported per kernel.
+    xu_theory = 148 * 8 * OPS_PER_PAIR * sm_mhz * 1e6 / 1e12
+    for k in per_kernel.values():
+        k["frac_xu_theoretical"] = k["TOps_s"] / xu_theory
     roofline = None
     if dominant:
         roofline = {"bound": "alu", "kernel": dominant, "achieved": per_kernel[dominant]["TOps_s"],
-                    "peak": xu_peak, "unit": "TOps/s", "frac": per_kernel[dominant]["frac_xu_sincos"],
+                    "peak": xu_theory, "unit": "TOps/s", "frac": per_kernel[dominant]["TOps_s"] / xu_theory,
                     "traffic": traffic,
-                    "peak_source": "measured sincos throughput of the XU/MUFU pipe (idg_rho_benchmark rho=0) "
-                                   "x 36 paper-ops per pair, this process: the sincos roofline of a kernel "
-                                   "that evaluates one sincos per (pixel, visibility) pair (the paper's "
-                                   "kernels, the degridder); kernels['gridder'] reports its own bound "
-                                   "(fewer sincos per pair by accumulator rotation) as peak_own_TOps_s",
+                    "peak_source": "one-sincos-per-pair roofline from unit counts at the timed region's SM clock: "
+                                   "148 SMs x 16 MUFU lanes/clk / 2 (sin + cos) x 36 paper-ops per pair "
+                                   "(P:258, P:276); the paper's formulation cannot exceed it.  The B200 kernels "
+                                   "evaluate 0.125-0.5 sincos per pair (rotation), so their own sincos bound "
+                                   "(kernels[*].peak_own_TOps_s) is higher; what binds them is instruction issue "
+                                   "(see DESIGN.md section 7)",
+                    "peak_measured_xu": xu_peak, "frac_measured_xu": per_kernel[dominant]["frac_xu_sincos"],
+                    "peak_measured_xu_source": "measured sincos throughput of the XU/MUFU pipe "
+                                               "(idg_rho_benchmark rho=0, best of 3) x 36, this process",
                     "variant": per_kernel[dominant]["variant"],
                     "peak_rho17": rho17, "frac_rho17": per_kernel[dominant]["frac_rho17"],
                     "peak_rho17_source": "paper's modified roofline: FMA:sincos mix at rho=17 (P:276-290), "
                                          "measured in this process",
-                    "peak_theoretical_xu": 148 * 8 * OPS_PER_PAIR * sm_mhz * 1e6 / 1e12,
                     "ops_per_pair": OPS_PER_PAIR, "pairs_per_launch": pairs,
                     "clocks_during_peak": rclocks.summary()}
 
