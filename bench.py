@@ -228,10 +228,18 @@ def run_ours(args):
         _build.build()
 
     rank, world, local = dist_env()
+    # IDG_BENCH_SHARED_GPU=1 (testing only): every rank on cuda:0 over gloo, to exercise the multi-rank
+    # path (sharding, collectives, max-over-ranks timing) on a one-GPU box; NCCL refuses duplicate GPUs.
+    shared_gpu = os.environ.get("IDG_BENCH_SHARED_GPU") == "1"
+    if shared_gpu:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if shared_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
 
     over = {"T": args.timesteps} if args.timesteps else {}
     full = idgsynth.make_observation(args.config, **over)
