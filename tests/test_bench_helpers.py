@@ -1,0 +1,26 @@
+"""bench.py host helpers (no GPU): sincos-per-pair accounting of each kernel family and the
+one-line JSON contract of the reference arm's shape."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import bench  # noqa: E402
+
+
+def test_sincos_per_pair_by_family():
+    spp = bench.sincos_per_pair
+    assert spp("gridder_tc<24,W12,MT3,minB2>", 16) == 1.0          # the paper's one sincos per pair
+    assert spp("degridder_tc<24,W8,MT2,minB4>", 16) == 1.0
+    assert spp("gridder_rot2<24,W12,MT3,minB2,KPT2>", 16) == 0.5     # group-0 phasors only
+    assert spp("gridder_rot2<32,W16,MT4,minB2,KPT4,GP2>", 32) == 0.25
+    assert spp("gridder_rot<24,W12,MT3,minB2,KPT4>", 16) == 0.75     # + E_t per lane
+    assert spp("degridder_rot<24,W8,minB4,U1,C16>", 16) == 0.5       # row 0 + E for 4 rows
+    assert spp("degridder_rot8<24,W8,minB2,U1,C16>", 16) == 0.25
+    assert spp("degridder_rot16<24,W4,minB3,U4,C16>", 16) == 0.125
+
+
+def test_ops_per_pair_is_the_papers():
+    # 17 FMA + 1 sincos = 36 paper-ops per (pixel, visibility) pair
+    assert bench.OPS_PER_PAIR == 36
