@@ -710,7 +710,7 @@ __device__ __forceinline__ f2p add2(f2p a, f2p b) {
     return r;
 }
 
-template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB, int TU = 1>
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB, int TU = 1, int NSM = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const KernelArgs a) {
     constexpr int NT = WARPS * 32;
     constexpr int NPIX = NS * NS;
@@ -725,6 +725,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
     float4 *raw_s = reinterpret_cast<float4 *>(smem);                // [VB][2]
     uint4 *frag_s = reinterpret_cast<uint4 *>(raw_s + 2 * VB);       // [KBB][32]
     float4 *coef_s = reinterpret_cast<float4 *>(frag_s + KBB * 32);  // [TPB][2]
+    f2p *n_s = reinterpret_cast<f2p *>(coef_s + 2 * (KBB + 1));     // NSM: [NPIX / 16][8] n of rows (g, g+8)
     __shared__ float red_s[WARPS];
 
     const int item = a.order[blockIdx.x];
@@ -752,6 +753,13 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
         pl[i] = pk(l2[0], l2[1]);
         pm[i] = pk(m2[0], m2[1]);
         pn[i] = pk(n2[0], n2[1]);
+        // NSM: the w-term n lives in shared memory (8 fewer live registers per tile pair at N~ = 32)
+        if (NSM && q == 0) n_s[(warp * MT + i) * 8 + g] = pn[i];
+        if (NSM == 2 && q == 0) {   // NSM = 2: l and m as well, after the n pairs: [NPIX / 16][8] {l pair, m pair}
+            f2p *lm = n_s + NPIX / 2 + ((warp * MT + i) * 8 + g) * 2;
+            lm[0] = pl[i];
+            lm[1] = pm[i];
+        }
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
     }
@@ -822,8 +830,18 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
                 uint4 bf0[GP];   // B fragments of the first pass, loaded ahead of the sincos
 #pragma unroll
                 for (int j = 0; j < GP; ++j) bf0[j] = fr[j * 32];
-                const float2 ph0 = unpk(fma2(dup(c0u), pl[i], fma2(dup(c0v), pm[i], mul2(dup(c0w), pn[i]))));
-                const float2 ph1 = unpk(fma2(dup(c4u), pl[i], fma2(dup(c4v), pm[i], mul2(dup(c4w), pn[i]))));
+                f2p nv = pn[i], lv = pl[i], mv = pm[i];
+                if constexpr (NSM) {
+                    // re-read every timestep (volatile: not hoisted into registers, which is the point)
+                    const uint32_t addr = uint32_t(__cvta_generic_to_shared(n_s + (warp * MT + i) * 8 + g));
+                    asm volatile("ld.shared.b64 %0, [%1];" : "=l"(nv) : "r"(addr));
+                    if constexpr (NSM == 2) {
+                        const uint32_t a2 = uint32_t(__cvta_generic_to_shared(n_s + NPIX / 2 + ((warp * MT + i) * 8 + g) * 2));
+                        asm volatile("ld.shared.v2.b64 {%0, %1}, [%2];" : "=l"(lv), "=l"(mv) : "r"(a2));
+                    }
+                }
+                const float2 ph0 = unpk(fma2(dup(c0u), lv, fma2(dup(c0v), mv, mul2(dup(c0w), nv))));
+                const float2 ph1 = unpk(fma2(dup(c4u), lv, fma2(dup(c4v), mv, mul2(dup(c4w), nv))));
                 float sn[4], cs[4];
                 __sincosf(ph0.x, &sn[0], &cs[0]);   // row g,   slot q
                 __sincosf(ph0.y, &sn[1], &cs[1]);   // row g+8, slot q
@@ -1483,15 +1501,15 @@ cudaError_t launch_gridder_rot(const KernelArgs &a, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int TU = 1>
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int TU = 1, int NSM = 0>
 cudaError_t launch_gridder_rot2(const KernelArgs &a, cudaStream_t st) {
     cudaError_t terr = ensure_dft_tables();
     if (terr != cudaSuccess) return terr;
-    const size_t smem = gridder_rot_smem_bytes(NS, KBB);
-    cudaError_t err = dev::prepare(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, TU>, smem);
+    const size_t smem = gridder_rot_smem_bytes(NS, KBB) + size_t(NSM) * NS * NS * 4 + (NSM == 2 ? size_t(NS) * NS * 4 : 0);
+    cudaError_t err = dev::prepare(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, TU, NSM>, smem);
     if (err != cudaSuccess) return err;
     LaunchScope scope("gridder", st);
-    gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, TU><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
+    gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, TU, NSM><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -1527,13 +1545,19 @@ cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
 #define TGROT2K(NS, W, MT, MB, KPT, KB) \
     {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",KB" #KB ">", \
      launch_gridder_rot2<NS, W, MT, MB, KPT, KPT, KB>, 8 * KPT}
+#define TGROT2N(NS, W, MT, MB, KPT, GP) \
+    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP ",nsm>", \
+     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, 1, 1>, 8 * KPT}
+#define TGROT2N2(NS, W, MT, MB, KPT, GP) \
+    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP ",lmnsm>", \
+     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, 1, 2>, 8 * KPT}
 #define TGROT2P(NS, W, MT, MB, KPT, GP) \
     {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP ">", \
      launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128>, 8 * KPT}
 const Variant kTcGridder[] = {
     TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
     TGROT2K(24, 12, 3, 2, 2, 64),
-    TGROT2P(32, 16, 4, 2, 4, 2), TGROT2(32, 16, 4, 1, 4), TGROT2P(32, 16, 4, 1, 4, 2), TGROT2P(32, 32, 2, 1, 4, 2), TGROT2(32, 32, 2, 1, 4), TGROT2(32, 16, 4, 2, 4), TGROT2(32, 16, 4, 2, 2), TGROT2(32, 16, 4, 1, 2), TGROT2(32, 32, 2, 1, 2), TGROT2(32, 16, 4, 2, 1),
+    TGROT2N(32, 16, 4, 2, 4, 2), TGROT2N2(32, 16, 4, 2, 2, 2), TGROT2N(32, 16, 4, 2, 2, 2), TGROT2N2(24, 12, 3, 2, 2, 2), TGROT2P(32, 16, 4, 2, 4, 2), TGROT2(32, 16, 4, 1, 4), TGROT2P(32, 16, 4, 1, 4, 2), TGROT2P(32, 32, 2, 1, 4, 2), TGROT2(32, 32, 2, 1, 4), TGROT2(32, 16, 4, 2, 4), TGROT2(32, 16, 4, 2, 2), TGROT2(32, 16, 4, 1, 2), TGROT2(32, 32, 2, 1, 2), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TGROT(24, 12, 3, 2, 4), TGROT(24, 12, 3, 2, 2), TGROT(24, 12, 3, 1, 2), TGROT(24, 12, 3, 1, 4),
     TGROT(32, 16, 4, 2, 4), TGROT(32, 16, 4, 1, 4), TGROT(32, 16, 4, 1, 2), TGROT(32, 8, 8, 1, 4), TGROT(32, 16, 4, 1, 8),
@@ -1553,6 +1577,8 @@ const Variant kTcGridder[] = {
 #undef TGROT
 #undef TGROT2
 #undef TGROT2P
+#undef TGROT2N
+#undef TGROT2N2
 #undef TGROT2K
 #undef TG
 template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int TFL = 0>
