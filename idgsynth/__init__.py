@@ -82,6 +82,24 @@ class Observation:
             uvw=np.ascontiguousarray(self.uvw[baseline_begin:baseline_begin + nb, :nt]),
             aterm_offsets=np.asarray(offs, dtype=np.int32))
 
+    def select(self, baselines, nr_timesteps: int | None = None, time_begin: int = 0) -> "Observation":
+        """Any baselines (index list) over timesteps [time_begin, time_begin + nr_timesteps), with the SAME
+        L, N, taper, stations (A-term rows) etc.; A-term slot boundaries are cut to the window."""
+        idx = np.asarray(baselines, dtype=np.int64).reshape(-1)
+        nt = self.nr_timesteps - time_begin if nr_timesteps is None else nr_timesteps
+        t1 = time_begin + nt
+        offs = [0] + [o - time_begin for o in self.aterm_offsets.tolist() if time_begin < o < t1] + [nt]
+        return dataclasses.replace(
+            self, name=f"{self.name}[bl{idx.tolist()},t{time_begin}+{nt}]",
+            baselines=np.ascontiguousarray(self.baselines[idx]),
+            uvw=np.ascontiguousarray(self.uvw[idx, time_begin:t1]),
+            aterm_offsets=np.asarray(offs, dtype=np.int32))
+
+    def longest_baselines(self, k: int) -> np.ndarray:
+        """Indices of the k baselines reaching the largest |u|, |v| (the outer grid: |u| L near N/2)."""
+        r = np.max(np.abs(self.uvw[:, :, :2]), axis=(1, 2))
+        return np.sort(np.argsort(r)[::-1][:k])
+
 
 # ----------------------------------------------------------------------------------------------
 # station layouts (ENU metres)
@@ -182,7 +200,7 @@ def make_observation(name: str, **overrides) -> Observation:
     aterms, dt, w_offset, seed, ...) -- same recipe, same seed unless overridden."""
     cfg = dict(CONFIGS[name])
     for k, v in overrides.items():
-        if k not in cfg and k not in ("w_offset", "C_block", "w_planes"):
+        if k not in cfg and k not in ("w_offset", "C_block", "w_planes", "channels"):
             raise KeyError(k)
         cfg[k] = v
     rng = np.random.default_rng(cfg["seed"])
@@ -204,6 +222,13 @@ def make_observation(name: str, **overrides) -> Observation:
     T = cfg["T"]
     uvw = earth_rotation_uvw(xyz, bl, T, cfg["dt"], math.radians(cfg["dec"]))
     freqs = cfg["f0"] + cfg["df"] * np.arange(cfg["C"], dtype=np.float64)
+    if cfg.get("channels", "uniform") == "gap_jitter":
+        # a real channel table: one channel missing (flagged / split band) and +-1 kHz jitter, so the
+        # spacing is not uniform and the kernels that rotate phasors across channels may not be used
+        full = cfg["f0"] + cfg["df"] * np.arange(cfg["C"] + 1, dtype=np.float64)
+        full = np.delete(full, (cfg["C"] + 1) // 3)
+        jit = np.random.default_rng(cfg["seed"] + 17).uniform(-1e3, 1e3, cfg["C"])
+        freqs = full + jit
     L = image_size_for(uvw, freqs, cfg["N"], cfg["Ns"])
     slot = cfg["slot"]
     offs = np.asarray(list(range(0, T, slot)) + [T], dtype=np.int32)
@@ -262,13 +287,20 @@ def _grdsf(nu: np.ndarray) -> np.ndarray:
 
 
 def make_taper(subgrid_size: int, kind: str = "spheroidal") -> np.ndarray:
-    """float32 [N~][N~] image-domain taper (the 'spheroidal'); separable, positive, peak 1."""
+    """float32 [N~][N~] = taper[y][x], the image-domain taper (the 'spheroidal'); separable,
+    positive, peak 1.  kind="asymmetric" tilts it along x only (s(y) s(x) (1 + 0.2 x')), so that a
+    [y][x] <-> [x][y] slip anywhere (oracle or kernels) changes the result."""
     n = subgrid_size
     if kind == "ones":
         return np.ones((n, n), dtype=np.float32)
     nu = np.abs(np.arange(n) - n / 2) / (n / 2 + 1)
     s = _grdsf(nu) * (1 - nu * nu)
     s = s / s.max()
+    if kind == "asymmetric":
+        xx = (np.arange(n) - n / 2) / (n / 2)
+        return np.outer(s, s * (1 + 0.2 * xx)).astype(np.float32)
+    if kind != "spheroidal":
+        raise ValueError(kind)
     return np.outer(s, s).astype(np.float32)
 
 

@@ -26,9 +26,8 @@ idg_status fail(idg_status st, const std::string &msg) {
     return st;
 }
 
-idg_status cuda_fail(cudaError_t e, const char *what) {
-    return fail(IDG_ERR_CUDA, std::string(what) + ": " + cudaGetErrorName(e) + " (" +
-                                  cudaGetErrorString(e) + ")");
+idg_status cuda_fail(cudaError_t e, const std::string &what) {
+    return fail(IDG_ERR_CUDA, what + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")");
 }
 
 std::atomic<int64_t> g_launches{0};
@@ -45,15 +44,28 @@ std::map<std::string, std::pair<int64_t, double>> g_prof_totals;
 constexpr int kStagingBuffers = 3;                  // triple buffering (Fig. 7)
 constexpr size_t kHostChunkBytes = size_t(128) << 20;  // visibilities per work group (host-streamed calls)
 
+// Events of the host-streamed pipeline for one workspace (its staging buffers), grown on demand.
+struct PipeEvents {
+    cudaEvent_t entry = nullptr;                              // the caller's stream at call entry
+    std::vector<cudaEvent_t> h2d, kernel_g, kernel_d, d2h;    // per staging buffer
+    ~PipeEvents() {
+        if (entry) cudaEventDestroy(entry);
+        for (auto *v : {&h2d, &kernel_g, &kernel_d, &d2h})
+            for (cudaEvent_t ev : *v) cudaEventDestroy(ev);
+    }
+};
+
 struct DeviceCopy {
     idg_metadata *items = nullptr;
     int32_t *order = nullptr;      // launch order of the device-resident calls (largest work first)
     int32_t *iota = nullptr;       // plan order (work groups of the host-streamed calls)
     int32_t *baselines = nullptr;
     double *frequencies = nullptr;
-    // host-streamed pipeline: one copy stream per direction + per-buffer events (grown on demand)
+    int64_t *dropped = nullptr;    // [nr][2] (visibility offset, count) of the dropped visibilities
+    // host-streamed pipeline: one copy stream per direction + events per workspace (keyed by its address,
+    // so calls on different workspaces never wait on each other's buffers)
     cudaStream_t h2d = nullptr, d2h = nullptr;
-    std::vector<cudaEvent_t> *ev_h2d = nullptr, *ev_kernel_g = nullptr, *ev_kernel_d = nullptr, *ev_d2h = nullptr;
+    std::map<const void *, std::unique_ptr<PipeEvents>> *pipes = nullptr;
     std::mutex *pipeline_mu = nullptr;
 };
 
@@ -62,6 +74,7 @@ struct DeviceCopy {
 struct WorkGroup {
     int32_t b0, b1;
     int64_t i0, i1;
+    int64_t r0, r1;   // its dropped-visibility ranges [r0, r1) (indices into idg_plan::dropped)
 };
 
 bool supported_subgrid(int32_t n) { return n == 16 || n == 24 || n == 32; }
@@ -79,6 +92,8 @@ struct idg_plan {
     int64_t nr_vis_assigned = 0, nr_vis_dropped = 0, nr_pairs = 0;
     int32_t max_channels_in_item = 0;
     int32_t max_timesteps_in_item = 0;
+    std::vector<int64_t> dropped;    // [nr][2]: (offset, count) in visibilities of every dropped run,
+                                     // split at baseline boundaries (R-12, R-13: predicted as 0)
     std::vector<WorkGroup> groups;   // host-streamed work groups
     size_t group_bytes = 0;          // largest work group's visibility bytes
     int32_t channel_gcd = 1;
@@ -95,13 +110,10 @@ struct idg_plan {
             cudaFree(kv.second.items);
             cudaFree(kv.second.order);
             cudaFree(kv.second.iota);
+            cudaFree(kv.second.dropped);
+            delete kv.second.pipes;
             if (kv.second.h2d) cudaStreamDestroy(kv.second.h2d);
             if (kv.second.d2h) cudaStreamDestroy(kv.second.d2h);
-            for (auto *v : {kv.second.ev_h2d, kv.second.ev_kernel_g, kv.second.ev_kernel_d, kv.second.ev_d2h}) {
-                if (!v) continue;
-                for (cudaEvent_t ev : *v) cudaEventDestroy(ev);
-                delete v;
-            }
             delete kv.second.pipeline_mu;
             cudaFree(kv.second.baselines);
             cudaFree(kv.second.frequencies);
@@ -130,7 +142,7 @@ struct idg_plan {
         DeviceCopy dc;
         auto release = [&dc]() {  // undo a partial device copy
             cudaFree(dc.items); cudaFree(dc.order); cudaFree(dc.iota); cudaFree(dc.baselines);
-            cudaFree(dc.frequencies);
+            cudaFree(dc.frequencies); cudaFree(dc.dropped);
             if (dc.h2d) cudaStreamDestroy(dc.h2d);
             if (dc.d2h) cudaStreamDestroy(dc.d2h);
         };
@@ -139,7 +151,8 @@ struct idg_plan {
             (e = cudaMalloc(&dc.order, ni * sizeof(int32_t))) != cudaSuccess ||
             (e = cudaMalloc(&dc.iota, ni * sizeof(int32_t))) != cudaSuccess ||
             (e = cudaMalloc(&dc.baselines, std::max<size_t>(2, baselines.size()) * 4)) != cudaSuccess ||
-            (e = cudaMalloc(&dc.frequencies, frequencies.size() * 8)) != cudaSuccess) {
+            (e = cudaMalloc(&dc.frequencies, frequencies.size() * 8)) != cudaSuccess ||
+            (!dropped.empty() && (e = cudaMalloc(&dc.dropped, dropped.size() * 8)) != cudaSuccess)) {
             release();
             return e == cudaErrorMemoryAllocation ? fail(IDG_ERR_OUT_OF_MEMORY, "plan device copy")
                                                   : cuda_fail(e, "cudaMalloc(plan)");
@@ -152,7 +165,9 @@ struct idg_plan {
               (e = cudaMemcpy(dc.iota, iota.data(), iota.size() * sizeof(int32_t), cudaMemcpyHostToDevice)) != cudaSuccess)) ||
             (!baselines.empty() &&
              (e = cudaMemcpy(dc.baselines, baselines.data(), baselines.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess) ||
-            (e = cudaMemcpy(dc.frequencies, frequencies.data(), frequencies.size() * 8, cudaMemcpyHostToDevice)) != cudaSuccess) {
+            (e = cudaMemcpy(dc.frequencies, frequencies.data(), frequencies.size() * 8, cudaMemcpyHostToDevice)) != cudaSuccess ||
+            (!dropped.empty() &&
+             (e = cudaMemcpy(dc.dropped, dropped.data(), dropped.size() * 8, cudaMemcpyHostToDevice)) != cudaSuccess)) {
             release();
             return cuda_fail(e, "cudaMemcpy(plan)");
         }
@@ -161,10 +176,7 @@ struct idg_plan {
             release();
             return cuda_fail(e, "cudaStreamCreate(pipeline)");
         }
-        dc.ev_h2d = new std::vector<cudaEvent_t>();
-        dc.ev_kernel_g = new std::vector<cudaEvent_t>();
-        dc.ev_kernel_d = new std::vector<cudaEvent_t>();
-        dc.ev_d2h = new std::vector<cudaEvent_t>();
+        dc.pipes = new std::map<const void *, std::unique_ptr<PipeEvents>>();
         dc.pipeline_mu = new std::mutex();
         auto res = device.emplace(dev, dc);
         *out = &res.first->second;
@@ -233,15 +245,53 @@ int staging_buffers(const idg_plan *plan, size_t workspace_bytes) {
     const size_t per_dir = workspace_bytes / (2 * plan->group_bytes);
     return int(std::max<size_t>(kStagingBuffers, std::min<size_t>(per_dir, plan->groups.size())));
 }
-cudaError_t ensure_events(const DeviceCopy *dc, int n) {
-    for (auto *v : {dc->ev_h2d, dc->ev_kernel_g, dc->ev_kernel_d, dc->ev_d2h})
+// The pipeline events of workspace `ws` with at least n per-buffer events (pipeline_mu held).
+cudaError_t pipe_events(const DeviceCopy *dc, const void *ws, int n, PipeEvents **out) {
+    auto &slot = (*dc->pipes)[ws];
+    if (!slot) slot.reset(new PipeEvents());
+    PipeEvents *pe = slot.get();
+    cudaError_t e = cudaSuccess;
+    if (!pe->entry && (e = cudaEventCreateWithFlags(&pe->entry, cudaEventDisableTiming)) != cudaSuccess) return e;
+    for (auto *v : {&pe->h2d, &pe->kernel_g, &pe->kernel_d, &pe->d2h})
         while (int(v->size()) < n) {
             cudaEvent_t ev;
-            cudaError_t e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
-            if (e != cudaSuccess) return e;
+            if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess) return e;
             v->push_back(ev);
         }
+    *out = pe;
     return cudaSuccess;
+}
+
+// Zero the dropped visibilities [r0, r1) of the plan's range list in `vis` (whose first element is
+// visibility `base` of the full array) on stream s.
+cudaError_t zero_dropped(const DeviceCopy *dc, void *vis, int64_t base, int64_t r0, int64_t r1, cudaStream_t s) {
+    if (r1 <= r0) return cudaSuccess;
+    return idg::launch_zero_ranges(static_cast<float2 *>(vis), dc->dropped + 2 * r0, r1 - r0, base, s);
+}
+
+// The runs of visibilities no item covers (R-12, R-13), per baseline, as (offset, count) pairs.
+void dropped_ranges(const std::vector<idg_metadata> &items, int32_t nbl, int32_t T, int32_t C,
+                    std::vector<int64_t> &out) {
+    const int64_t per = int64_t(T) * C;
+    std::vector<uint8_t> cov(size_t(per), 0);
+    size_t it = 0;
+    for (int32_t b = 0; b < nbl; ++b) {
+        std::fill(cov.begin(), cov.end(), uint8_t(0));
+        for (; it < items.size() && items[it].baseline == b; ++it) {
+            const idg_metadata &m = items[it];
+            for (int32_t t = m.time_offset; t < m.time_offset + m.nr_timesteps; ++t)
+                std::fill(cov.begin() + int64_t(t) * C + m.channel_begin, cov.begin() + int64_t(t) * C + m.channel_end,
+                          uint8_t(1));
+        }
+        for (int64_t i = 0; i < per;) {
+            if (cov[size_t(i)]) { ++i; continue; }
+            int64_t j = i;
+            while (j < per && !cov[size_t(j)]) ++j;
+            out.push_back(int64_t(b) * per + i);
+            out.push_back(j - i);
+            i = j;
+        }
+    }
 }
 
 idg::KernelArgs make_args(const idg_plan *plan, const DeviceCopy *dc, const float *d_uvw,
@@ -373,18 +423,23 @@ idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, i
             plan->channels_uniform = uni ? 1 : 0;
             plan->channel_step = float(d0 / idg::kSpeedOfLight);
         }
+        if (plan->nr_vis_dropped > 0)
+            dropped_ranges(plan->items, nr_baselines, nr_timesteps, nr_channels, plan->dropped);
         // host-streamed work groups: contiguous baseline ranges of <= kHostChunkBytes visibilities
         {
             const size_t bl_bytes = size_t(nr_timesteps) * nr_channels * 32;
             size_t chunk = kHostChunkBytes;
             if (const char *env = std::getenv("IDG_HOST_CHUNK_BYTES")) chunk = std::max<size_t>(1, std::strtoull(env, nullptr, 10));
             const int32_t per = int32_t(std::max<size_t>(1, chunk / std::max<size_t>(1, bl_bytes)));
-            int64_t it = 0;
+            int64_t it = 0, r = 0;
+            const int64_t nr = int64_t(plan->dropped.size() / 2);
+            const int64_t vis_per_bl = int64_t(nr_timesteps) * nr_channels;
             for (int32_t b0 = 0; b0 < nr_baselines; b0 += per) {
                 const int32_t b1 = std::min(nr_baselines, b0 + per);
-                const int64_t i0 = it;
+                const int64_t i0 = it, r0 = r;
                 while (it < int64_t(plan->items.size()) && plan->items[it].baseline < b1) ++it;
-                plan->groups.push_back(WorkGroup{b0, b1, i0, it});
+                while (r < nr && plan->dropped[2 * r] < int64_t(b1) * vis_per_bl) ++r;
+                plan->groups.push_back(WorkGroup{b0, b1, i0, it, r0, r});
                 plan->group_bytes = std::max(plan->group_bytes, size_t(b1 - b0) * bl_bytes);
             }
         }
@@ -471,19 +526,22 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
     try {
         if (!plan) return fail(IDG_ERR_INVALID_ARG, "plan is NULL");
         const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-        if (plan->nr_vis_dropped > 0 || plan->items.empty()) {
-            // dropped visibilities are defined as 0 (R-12, R-13); items overwrite the rest
-            if (!d_vis) return fail(IDG_ERR_INVALID_ARG, "d_vis is NULL");
+        if (plan->items.empty()) {
+            // nothing to predict: every visibility is dropped and defined as 0 (R-12, R-13)
             const size_t bytes = size_t(plan->nr_baselines) * plan->nr_timesteps * plan->nr_channels * 32;
-            cudaError_t e = cudaMemsetAsync(d_vis, 0, bytes, s);
-            if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(vis)");
+            if (bytes > 0 && !d_vis) return fail(IDG_ERR_INVALID_ARG, "d_vis is NULL");
+            cudaError_t e = bytes > 0 ? cudaMemsetAsync(d_vis, 0, bytes, s) : cudaSuccess;
+            return e == cudaSuccess ? IDG_OK : cuda_fail(e, "cudaMemsetAsync(vis)");
         }
         idg_status st = validate_call(plan, d_vis, d_uvw, d_aterms, d_taper, d_grid);
-        if (st != IDG_OK || plan->items.empty()) return st;
+        if (st != IDG_OK) return st;
         const DeviceCopy *dc = nullptr;
         if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        // dropped visibilities are 0 (R-12, R-13): only their runs are written; the items overwrite the rest
+        cudaError_t e = zero_dropped(dc, d_vis, 0, 0, int64_t(plan->dropped.size() / 2), s);
+        if (e != cudaSuccess) return cuda_fail(e, "zero dropped visibilities");
         idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper, d_vis, const_cast<void *>(d_grid));
-        cudaError_t e = idg::launch_degridder(a, s);
+        e = idg::launch_degridder(a, s);
         if (e != cudaSuccess) return cuda_fail(e, "degridder launch");
         return IDG_OK;
     } catch (const std::exception &ex) {
@@ -496,6 +554,15 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
 // groups (contiguous baseline ranges) stream through kStagingBuffers device buffers; uploads run on a
 // copy stream, downloads on another, kernels on the caller's stream, ordered with events.
 // ------------------------------------------------------------------------------------------------
+// A failing event call inside the pipeline is reported like a failing copy or launch.
+#define IDG_PIPE(call)                      \
+    do {                                    \
+        if ((e = (call)) != cudaSuccess) {  \
+            what = #call;                   \
+            goto pipe_error;                \
+        }                                   \
+    } while (0)
+
 idg_status idg_grid_host(const idg_plan *plan, const void *h_vis, const float *d_uvw, const void *d_aterms,
                          const float *d_taper, void *d_grid, void *d_workspace, size_t workspace_bytes,
                          idg_stream stream) {
@@ -514,30 +581,37 @@ idg_status idg_grid_host(const idg_plan *plan, const void *h_vis, const float *d
         const int64_t bl_f2 = int64_t(plan->nr_timesteps) * plan->nr_channels * 4;  // float2 per baseline
         const int nb = staging_buffers(plan, workspace_bytes);
         char *staging = static_cast<char *>(d_workspace);                        // grid half of the workspace
-        cudaError_t e = ensure_events(dc, nb);
-        for (size_t gi = 0; gi < plan->groups.size() && e == cudaSuccess; ++gi) {
+        const char *what = "";
+        PipeEvents *pe = nullptr;
+        cudaError_t e = pipe_events(dc, d_workspace, nb, &pe);
+        if (e != cudaSuccess) return cuda_fail(e, "idg_grid_host: events");
+        // the uploads read h_vis and overwrite the staging buffers: both may still be in use by work the
+        // caller queued on `stream` before this call (a copy into h_vis, a kernel on a recycled workspace)
+        IDG_PIPE(cudaEventRecord(pe->entry, s));
+        IDG_PIPE(cudaStreamWaitEvent(dc->h2d, pe->entry, 0));
+        for (size_t gi = 0; gi < plan->groups.size(); ++gi) {
             const WorkGroup &g = plan->groups[gi];
             const int b = int(gi % nb);
             char *buf = staging + size_t(b) * plan->group_bytes;
             // the buffer is free once the gridder that last read it has finished
             // (also across calls: an event never recorded is complete)
-            cudaStreamWaitEvent(dc->h2d, (*dc->ev_kernel_g)[b], 0);
-            e = cudaMemcpyAsync(buf, static_cast<const char *>(h_vis) + size_t(g.b0) * bl_bytes,
-                                size_t(g.b1 - g.b0) * bl_bytes, cudaMemcpyHostToDevice, dc->h2d);
-            if (e != cudaSuccess) break;
-            cudaEventRecord((*dc->ev_h2d)[b], dc->h2d);
-            cudaStreamWaitEvent(s, (*dc->ev_h2d)[b], 0);
+            IDG_PIPE(cudaStreamWaitEvent(dc->h2d, pe->kernel_g[b], 0));
+            IDG_PIPE(cudaMemcpyAsync(buf, static_cast<const char *>(h_vis) + size_t(g.b0) * bl_bytes,
+                                     size_t(g.b1 - g.b0) * bl_bytes, cudaMemcpyHostToDevice, dc->h2d));
+            IDG_PIPE(cudaEventRecord(pe->h2d[b], dc->h2d));
+            IDG_PIPE(cudaStreamWaitEvent(s, pe->h2d[b], 0));
             if (g.i1 > g.i0) {
                 idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper,
                                               reinterpret_cast<float2 *>(buf) - int64_t(g.b0) * bl_f2, d_grid);
                 a.order = dc->iota + g.i0;
                 a.nr_items = g.i1 - g.i0;
-                e = idg::launch_gridder(a, s);
+                IDG_PIPE(idg::launch_gridder(a, s));
             }
-            cudaEventRecord((*dc->ev_kernel_g)[b], s);
+            IDG_PIPE(cudaEventRecord(pe->kernel_g[b], s));
         }
-        if (e != cudaSuccess) return cuda_fail(e, "idg_grid_host");
         return IDG_OK;
+    pipe_error:
+        return cuda_fail(e, std::string("idg_grid_host: ") + what);
     } catch (const std::exception &ex) {
         return fail(IDG_ERR_INVALID_ARG, ex.what());
     }
@@ -550,9 +624,15 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
         idg_status st = validate_call(plan, h_vis, d_uvw, d_aterms, d_taper, d_grid);
         if (st != IDG_OK) return st;
         const size_t bl_bytes = size_t(plan->nr_timesteps) * plan->nr_channels * 32;
-        if (plan->items.empty()) {  // nothing to predict: every visibility is dropped -> 0 (no GPU work)
+        const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+        if (plan->items.empty()) {  // nothing to predict: every visibility is dropped -> 0
             const size_t bytes = size_t(plan->nr_baselines) * bl_bytes;
             if (bytes > 0 && !h_vis) return fail(IDG_ERR_INVALID_ARG, "h_vis is NULL");
+            // ordered after the caller's work on `stream` (which may still read h_vis), like the downloads
+            // (without a CUDA device there is no queued work to wait for)
+            cudaError_t e = cudaStreamSynchronize(s);
+            if (e == cudaErrorNoDevice || e == cudaErrorInsufficientDriver) e = cudaGetLastError(), e = cudaSuccess;
+            if (e != cudaSuccess) return cuda_fail(e, "idg_degrid_host: cudaStreamSynchronize");
             if (bytes > 0) std::memset(h_vis, 0, bytes);
             return IDG_OK;
         }
@@ -560,53 +640,53 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
         if (!d_workspace || workspace_bytes < need)
             return fail(IDG_ERR_WORKSPACE_TOO_SMALL, "host-streamed degridding needs idg_host_workspace_size() = " +
                                                          std::to_string(need) + " bytes");
-        const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
         const DeviceCopy *dc = nullptr;
         if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
         std::lock_guard<std::mutex> lock(*dc->pipeline_mu);
         const int64_t bl_f2 = int64_t(plan->nr_timesteps) * plan->nr_channels * 4;
+        const int64_t bl_vis = int64_t(plan->nr_timesteps) * plan->nr_channels;
         const int nb = staging_buffers(plan, workspace_bytes);
         char *staging = static_cast<char *>(d_workspace) + size_t(nb) * plan->group_bytes;
-        cudaError_t e = ensure_events(dc, nb);
+        const char *what = "";
+        PipeEvents *pe = nullptr;
+        cudaError_t e = pipe_events(dc, d_workspace, nb, &pe);
+        if (e != cudaSuccess) return cuda_fail(e, "idg_degrid_host: events");
         size_t last = 0;
-        for (size_t gi = 0; gi < plan->groups.size() && e == cudaSuccess; ++gi) {
+        for (size_t gi = 0; gi < plan->groups.size(); ++gi) {
             const WorkGroup &g = plan->groups[gi];
             const int b = int(gi % nb);
             char *buf = staging + size_t(b) * plan->group_bytes;
             const size_t bytes = size_t(g.b1 - g.b0) * bl_bytes;
             // the buffer is free once its previous download has finished
-            cudaStreamWaitEvent(s, (*dc->ev_d2h)[b], 0);
-            if (plan->nr_vis_dropped > 0) {
-                e = cudaMemsetAsync(buf, 0, bytes, s);  // dropped visibilities are 0 (R-12, R-13)
-                if (e != cudaSuccess) break;
-            }
+            IDG_PIPE(cudaStreamWaitEvent(s, pe->d2h[b], 0));
+            // dropped visibilities are 0 (R-12, R-13): only their runs are written, the items overwrite the rest
+            IDG_PIPE(zero_dropped(dc, buf, int64_t(g.b0) * bl_vis, g.r0, g.r1, s));
             if (g.i1 > g.i0) {
                 idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper,
                                               reinterpret_cast<float2 *>(buf) - int64_t(g.b0) * bl_f2,
                                               const_cast<void *>(d_grid));
                 a.order = dc->iota + g.i0;
                 a.nr_items = g.i1 - g.i0;
-                e = idg::launch_degridder(a, s);
-                if (e != cudaSuccess) break;
-            } else if (plan->nr_vis_dropped == 0) {
-                e = cudaMemsetAsync(buf, 0, bytes, s);
-                if (e != cudaSuccess) break;
+                IDG_PIPE(idg::launch_degridder(a, s));
             }
-            cudaEventRecord((*dc->ev_kernel_d)[b], s);
-            cudaStreamWaitEvent(dc->d2h, (*dc->ev_kernel_d)[b], 0);
-            e = cudaMemcpyAsync(static_cast<char *>(h_vis) + size_t(g.b0) * bl_bytes, buf, bytes,
-                                cudaMemcpyDeviceToHost, dc->d2h);
-            cudaEventRecord((*dc->ev_d2h)[b], dc->d2h);
+            // (the downloads start after all of the caller's earlier work on `stream`, which may read h_vis)
+            IDG_PIPE(cudaEventRecord(pe->kernel_d[b], s));
+            IDG_PIPE(cudaStreamWaitEvent(dc->d2h, pe->kernel_d[b], 0));
+            IDG_PIPE(cudaMemcpyAsync(static_cast<char *>(h_vis) + size_t(g.b0) * bl_bytes, buf, bytes,
+                                     cudaMemcpyDeviceToHost, dc->d2h));
+            IDG_PIPE(cudaEventRecord(pe->d2h[b], dc->d2h));
             last = gi;
         }
-        if (e != cudaSuccess) return cuda_fail(e, "idg_degrid_host");
         // completion of the call is observable on the caller's stream
-        for (int b = 0; b < nb && size_t(b) <= last; ++b) cudaStreamWaitEvent(s, (*dc->ev_d2h)[b], 0);
+        for (int b = 0; b < nb && size_t(b) <= last; ++b) IDG_PIPE(cudaStreamWaitEvent(s, pe->d2h[b], 0));
         return IDG_OK;
+    pipe_error:
+        return cuda_fail(e, std::string("idg_degrid_host: ") + what);
     } catch (const std::exception &ex) {
         return fail(IDG_ERR_INVALID_ARG, ex.what());
     }
 }
+#undef IDG_PIPE
 
 idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
                              double *seconds) {

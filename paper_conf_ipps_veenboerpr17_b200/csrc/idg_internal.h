@@ -54,26 +54,27 @@ struct KernelArgs {
 };
 
 using Launcher = cudaError_t (*)(const KernelArgs &, cudaStream_t);
+using SmemFn = size_t (*)(const KernelArgs &);
 constexpr int kSimt = 0, kTensor = 1;
 struct Variant {
     int ns;            // subgrid size
     int v;             // channels per thread (SIMT degridder) / channel multiple (tensor gridder); 0 = any
     int kind;          // kSimt | kTensor
-    int needs_uniform; // 1: requires uniformly spaced channels (phasor recurrence over channels)
+    int needs_uniform; // 1: requires uniformly spaced channels (phasor rotation over channels)
     const char *name;
     Launcher fn;
     int max_channels = 0;  // > 0: every item has at most this many channels (unrolled channel groups)
+    SmemFn smem = nullptr; // dynamic shared memory of a launch (the plan's items must fit the device)
 };
 // Tensor-core variants (idg_kernels_tc.cu); the first eligible one is the default.
 const Variant *tc_gridder_variants(int *n);     // split-f16 mma (idg_kernels_tc.cu)
 const Variant *tc_degridder_variants(int *n);
-const Variant *tf32_gridder_variants(int *n);   // split-tf32 mma (idg_kernels_tf32.cu)
-const Variant *umma_gridder_variants(int *n);   // tcgen05 / TMEM (idg_kernels_umma.cu)
-const Variant *tf32_degridder_variants(int *n);
 
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s);
 cudaError_t launch_degridder(const KernelArgs &a, cudaStream_t s);
 const char *variant_names(int which);
+// vis[r[2i] - base .. + r[2i+1]) = 0 for i < nr (the plan's dropped-visibility runs, R-12 / R-13)
+cudaError_t launch_zero_ranges(float2 *vis, const int64_t *ranges, int64_t nr, int64_t base, cudaStream_t s);
 const char *last_variant(int which);   // name of the variant the last launch used ("" before any)
 cudaError_t launch_rho_benchmark(int rho, int iterations, float *d_out, cudaStream_t s,
                                  int *blocks, int *threads, int *units_per_thread);

@@ -278,6 +278,11 @@ __global__ void __launch_bounds__(NT, MINB) degridder_kernel(const KernelArgs a)
     }
 }
 
+template <int NS>
+size_t smem_gridder_t(const KernelArgs &a) { return gridder_smem_bytes(NS, a.max_channels_in_item); }
+template <int NS>
+size_t smem_degridder_t(const KernelArgs &a) { return degridder_smem_bytes(NS, a.max_channels_in_item); }
+
 template <int NS, int P, int MINB>
 cudaError_t launch_gridder_t(const KernelArgs &a, cudaStream_t st) {
     constexpr int NT = NS * NS / P;
@@ -300,28 +305,44 @@ cudaError_t launch_degridder_t(const KernelArgs &a, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-// SIMT launch-shape variants (first entry per (NS, V) is the SIMT default; tuned with scripts/tune.py).
+// SIMT variants (the paper's kernel structure on the CUDA cores; launch shapes tuned with scripts/tune.py).
 // v = channels per thread for the degridder (every item's channel count must be a multiple of v).
-#define GV(NS, P, MB) {NS, 0, kSimt, 0, "gridder<" #NS ",P" #P ",minB" #MB ">", launch_gridder_t<NS, P, MB>}
-const Variant kGridderVariants[] = {
-    GV(24, 6, 4), GV(24, 6, 5), GV(24, 6, 6), GV(24, 3, 3), GV(24, 3, 4), GV(24, 2, 4), GV(24, 9, 3),
-    GV(32, 4, 2), GV(32, 8, 3), GV(32, 8, 4), GV(32, 4, 3), GV(32, 16, 4),
-    GV(16, 4, 4), GV(16, 4, 6), GV(16, 2, 4), GV(16, 8, 6),
-};
+#define GV(NS, P, MB) {NS, 0, kSimt, 0, "gridder<" #NS ",P" #P ",minB" #MB ">", launch_gridder_t<NS, P, MB>, 0, \
+                       smem_gridder_t<NS>}
+const Variant kGridderVariants[] = {GV(24, 6, 4), GV(32, 4, 2), GV(16, 4, 4)};
 #undef GV
-#define DV(NS, V, NT, MB) {NS, V, kSimt, 0, "degridder<" #NS ",V" #V ",T" #NT ",minB" #MB ">", launch_degridder_t<NS, V, NT, MB>}
-#define DV_ALL(NS) DV(NS, 8, 128, 4), DV(NS, 8, 128, 3), DV(NS, 8, 256, 1), DV(NS, 8, 256, 2), \
-    DV(NS, 8, 64, 6), DV(NS, 8, 64, 8), DV(NS, 4, 128, 4), DV(NS, 4, 256, 3), DV(NS, 4, 128, 6), \
-    DV(NS, 2, 128, 6), DV(NS, 1, 128, 6)
+#define DV(NS, V, NT, MB) {NS, V, kSimt, 0, "degridder<" #NS ",V" #V ",T" #NT ",minB" #MB ">", \
+                           launch_degridder_t<NS, V, NT, MB>, 0, smem_degridder_t<NS>}
+#define DV_ALL(NS) DV(NS, 8, 128, 4), DV(NS, 4, 128, 4), DV(NS, 2, 128, 6), DV(NS, 1, 128, 6)
 const Variant kDegridderVariants[] = {DV_ALL(24), DV_ALL(32), DV_ALL(16)};
 #undef DV_ALL
 #undef DV
+
+// Opt-in dynamic shared memory limit of the current device (cached per device).
+size_t max_dynamic_smem() {
+    static std::atomic<int> cache[64];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 0;
+    int v = cache[dev].load();
+    if (v == 0) {
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) return 0;
+        cache[dev].store(v);
+    }
+    return size_t(v);
+}
 
 bool eligible(const Variant &var, const KernelArgs &a) {
     if (var.ns != a.subgrid_size) return false;
     if (var.needs_uniform && !a.channels_uniform) return false;
     if (var.max_channels > 0 && a.max_channels_in_item > var.max_channels) return false;
-    return var.v == 0 || a.channel_gcd % var.v == 0;
+    if (var.v != 0 && a.channel_gcd % var.v != 0) return false;
+    // shared memory grows with the plan's largest item (T~ for the degridders, C~ for the gridders): a
+    // variant whose launch would not fit is skipped, so a kernel that fits (ultimately SIMT) runs instead
+    if (var.smem) {
+        const size_t lim = max_dynamic_smem();
+        if (lim > 0 && var.smem(a) > lim) return false;
+    }
+    return true;
 }
 
 // Variant choice.  Default: the first eligible tensor-core variant, else the first eligible SIMT
@@ -361,18 +382,12 @@ const std::vector<const Variant *> &tensor_variants(int which) {
             int n = 0;
             const Variant *t = tc_gridder_variants(&n);
             for (int i = 0; i < n; ++i) v.push_back(&t[i]);
-            t = tf32_gridder_variants(&n);
-            for (int i = 0; i < n; ++i) v.push_back(&t[i]);
-            t = umma_gridder_variants(&n);
-            for (int i = 0; i < n; ++i) v.push_back(&t[i]);
             return v;
         }(),
         [] {
             std::vector<const Variant *> v;
             int n = 0;
             const Variant *t = tc_degridder_variants(&n);
-            for (int i = 0; i < n; ++i) v.push_back(&t[i]);
-            t = tf32_degridder_variants(&n);
             for (int i = 0; i < n; ++i) v.push_back(&t[i]);
             return v;
         }()};
@@ -382,6 +397,24 @@ const std::vector<const Variant *> &tensor_variants(int which) {
 }  // namespace
 
 std::atomic<const char *> g_last_variant[2] = {"", ""};
+
+// Dropped visibilities are predicted as 0 (R-12, R-13): one CTA per run (grid-stride), 16-byte stores.
+__global__ void __launch_bounds__(256) zero_ranges_kernel(float4 *vis, const int64_t *ranges, int64_t nr,
+                                                          int64_t base) {
+    for (int64_t r = blockIdx.x; r < nr; r += gridDim.x) {
+        float4 *p = vis + 2 * (ranges[2 * r] - base);
+        const int64_t n = 2 * ranges[2 * r + 1];   // a visibility is 4 complex64 = 2 float4
+        for (int64_t i = threadIdx.x; i < n; i += blockDim.x) p[i] = make_float4(0.0f, 0.0f, 0.0f, 0.0f);
+    }
+}
+
+cudaError_t launch_zero_ranges(float2 *vis, const int64_t *ranges, int64_t nr, int64_t base, cudaStream_t s) {
+    if (nr <= 0) return cudaSuccess;
+    LaunchScope scope("zero_dropped", s);
+    const unsigned blocks = unsigned(std::min<int64_t>(nr, 148 * 16));
+    zero_ranges_kernel<<<blocks, 256, 0, s>>>(reinterpret_cast<float4 *>(vis), ranges, nr, base);
+    return cudaGetLastError();
+}
 
 cudaError_t launch_gridder(const KernelArgs &a, cudaStream_t s) {
     if (a.nr_items == 0) return cudaSuccess;

@@ -80,24 +80,6 @@ __device__ __forceinline__ void split2(float x, float y, uint32_t &hi, uint32_t 
 }
 __device__ __forceinline__ void split_phasor(float x, float y, uint32_t &hi, uint32_t &lo) { split2(x, y, hi, lo); }
 
-// (x, y) -> f16x2 hi = rn(x, y) and the exact fp32 residuals x - hi, y - hi (two FHFMA, no repacking):
-// the residuals feed a tf32 mma directly (it reads the top 19 bits of each fp32 register).
-__device__ __forceinline__ void split_hi_res(float x, float y, uint32_t &hi, float &dx, float &dy) {
-    hi = h2_bits(__floats2half2_rn(x, y));
-    asm("{\n.reg .f16 a, b, m;\nmov.b32 {a, b}, %2;\nmov.b16 m, 0xBC00;\n"
-        "fma.rn.f32.f16 %0, a, m, %3;\nfma.rn.f32.f16 %1, b, m, %4;\n}"
-        : "=f"(dx), "=f"(dy) : "r"(hi), "f"(x), "f"(y));
-}
-
-// D += A B, m16n8k8 tf32 (fp32 registers; A {(g, q), (g+8, q), (g, q+4), (g+8, q+4)}, B {(q, g), (q+4, g)}).
-__device__ __forceinline__ void mma1688_tf32(float (&d)[4], float a0, float a1, float a2, float a3, float b0,
-                                             float b1) {
-    asm("mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
-        "{%0,%1,%2,%3};"
-        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
-        : "r"(__float_as_uint(a0)), "r"(__float_as_uint(a1)), "r"(__float_as_uint(a2)), "r"(__float_as_uint(a3)),
-          "r"(__float_as_uint(b0)), "r"(__float_as_uint(b1)));
-}
 
 __device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
                                          uint32_t b0, uint32_t b1) {
@@ -307,10 +289,9 @@ inline size_t gridder_tc_smem_bytes(int NS, int max_channels, int kbb_ = kTcBatc
     return std::max(main, epi) + 16;
 }
 
-// REC = 1: channels are uniformly spaced, so the phasor of k-slot q+4 (channel c+4) is the phasor of
-// slot q times the per-(pixel, timestep) step exp(i 4 dnu/c Q_t): half of the sincos become one complex
-// multiply (4 FMA-pipe instructions) and the MUFU (XU) load per pair drops from 2 to ~1.25 (+ steps).
-template <int NS, int WARPS, int MT, int MINB, int REC, int KBB_ = kTcBatchKB>
+// The direct kernel: one sincos per (pixel, visibility) pair, any channel spacing (the fallback of the
+// rotation gridder for non-uniform channel tables and items of varying channel counts).
+template <int NS, int WARPS, int MT, int MINB, int KBB_ = kTcBatchKB>
 __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const KernelArgs a) {
     constexpr int NT = WARPS * 32;
     constexpr int NPIX = NS * NS;
@@ -393,8 +374,11 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
         // (4) f16 range: power-of-two scale from the batch maximum; never increase the running scale
         float mx = 0.0f;
         for (int i = threadIdx.x; i < 2 * nvb; i += NT) mx = abs_max4(raw_s[i], mx).x;
-        const float bscale = pow2_scale(block_max<WARPS>(mx, red_s));
-        if (cur_scale == 0.0f) {
+        // (an all-zero batch, e.g. flagged data, leaves the scale alone: it carries no range information)
+        const float bmax = block_max<WARPS>(mx, red_s);
+        const float bscale = bmax > 0.0f ? pow2_scale(bmax) : 0.0f;
+        if (bscale == 0.0f) {
+        } else if (cur_scale == 0.0f) {
             cur_scale = bscale;
         } else if (bscale < cur_scale) {
             const float f = bscale / cur_scale;  // exact power of two
@@ -432,16 +416,10 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
             // B_t, Q_t of both rows of every tile (packed pairs), once per timestep
             const float4 cB = coef_s[2 * (t - t_first)], cQ = coef_s[2 * (t - t_first) + 1];
             f2p Bv[MT], Qv[MT];
-            float stc[REC ? MT : 1][2], sts[REC ? MT : 1][2];
 #pragma unroll
             for (int i = 0; i < MT; ++i) {
                 Bv[i] = fma2(dup(cB.x), pl[i], fma2(dup(cB.y), pm[i], mul2(dup(cB.z), pn[i])));
                 Qv[i] = fma2(dup(cQ.x), pl[i], fma2(dup(cQ.y), pm[i], mul2(dup(cQ.z), pn[i])));
-                if (REC) {
-                    const float2 st = unpk(mul2(dup(4.0f * a.channel_step), Qv[i]));
-                    __sincosf(st.x, &sts[i][0], &stc[i][0]);
-                    __sincosf(st.y, &sts[i][1], &stc[i][1]);
-                }
             }
             const int k_begin = max(kb0, t * kpt), k_end = min(kb1, (t + 1) * kpt);
 #pragma unroll 1
@@ -456,17 +434,9 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
                     float sn[4], cs[4];
                     __sincosf(ph0.x, &sn[0], &cs[0]);
                     __sincosf(ph0.y, &sn[1], &cs[1]);
-                    if (REC) {  // slot q+4 = slot q x exp(i 4 dnu/c Q)
-#pragma unroll
-                        for (int r = 0; r < 2; ++r) {
-                            cs[2 + r] = fmaf(cs[r], stc[i][r], -sn[r] * sts[i][r]);
-                            sn[2 + r] = fmaf(cs[r], sts[i][r], sn[r] * stc[i][r]);
-                        }
-                    } else {
-                        const float2 ph1 = unpk(fma2(dq4, Qv[i], Bv[i]));  // (row g, row g+8) at slot q+4
-                        __sincosf(ph1.x, &sn[2], &cs[2]);
-                        __sincosf(ph1.y, &sn[3], &cs[3]);
-                    }
+                    const float2 ph1 = unpk(fma2(dq4, Qv[i], Bv[i]));  // (row g, row g+8) at slot q+4
+                    __sincosf(ph1.x, &sn[2], &cs[2]);
+                    __sincosf(ph1.y, &sn[3], &cs[3]);
 #pragma unroll
                     for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[i][j], al[i][j]);
                 }
@@ -500,196 +470,11 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_tc_kernel(const Kern
     gridder_epilogue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(tmp_s + 4 * NPIX), red_s);
 }
 
-// ------------------------------------------------------------------------------------------------
-// Tensor-core gridder with accumulator rotation across channel groups (uniformly spaced channels).
-//
-// The phase is linear in frequency (R-2: phi = B_t + (nu_c/c - f_ref) Q_t), so with channels
-// c = 8j + s (group j = 0..J-1, slot s = 0..7, J = C~/8) and spacing dnu,
-//     Phi(t, 8j + s) = Phi(t, s) E_t^j,    E_t = exp(i 8 dnu/c Q_t)    (per pixel and timestep)
-// and the per-timestep contribution to a pixel factorises:
-//     sum_c Phi(t,c) V(t,c) = sum_j E_t^j D_j,   D_j = sum_s Phi(t,s) V(t, 8j+s).
-// Every D_j is an mma of the SAME A fragment (the slot-s phasors of group 0) with group j's B fragment,
-// so the sincos + split work per (pixel, timestep) is that of 8 visibilities plus one sincos for E_t,
-// instead of C~.  D_j is formed fresh per timestep (split-f16, three products) and rotated into the
-// fp32 accumulator with E_t^j (E_t^j by recurrence).  Exact in exact arithmetic; the rounding is that of
-// one extra complex product per (pixel, timestep, group).  Batches hold whole timesteps.
-// ------------------------------------------------------------------------------------------------
 inline size_t gridder_rot_smem_bytes(int NS, int kbb_ = kTcBatchKB) {
     const size_t kbb = kbb_;
     const size_t main = kbb * 8 * 32 /*raw*/ + kbb * 32 * 16 /*frag*/ + (kbb + 1) * 32 /*coef*/;
     const size_t epi = size_t(2) * 4 * NS * NS * sizeof(float2) + size_t(NS) * NS * 16;  // sub_s, tmp_s, DFT table
     return std::max(main, epi) + 16;
-}
-
-template <int NS, int WARPS, int MT, int MINB, int KPT, int KBB_ = kTcBatchKB>
-__global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot_kernel(const KernelArgs a) {
-    constexpr int NT = WARPS * 32;
-    constexpr int NPIX = NS * NS;
-    static_assert(WARPS * MT * 16 == NPIX, "warps x m-tiles x 16 must cover the subgrid");
-    static_assert(KPT >= 1 && KPT <= KBB_, "channel groups per timestep");
-    constexpr int h = NS / 2;
-    constexpr int KBB = KBB_;
-    constexpr int VB = KBB * 8;
-    extern __shared__ __align__(16) unsigned char smem[];
-    float4 *raw_s = reinterpret_cast<float4 *>(smem);                // [VB][2]
-    uint4 *frag_s = reinterpret_cast<uint4 *>(raw_s + 2 * VB);       // [KBB][32]
-    float4 *coef_s = reinterpret_cast<float4 *>(frag_s + KBB * 32);  // [KBB+1][2]
-    __shared__ float red_s[WARPS];
-
-    const int item = a.order[blockIdx.x];
-    const ItemSetup s = dev::item_setup(a, item, NS);
-    const idg_metadata &md = s.md;
-    const int nc = s.nc;
-    const int kpt = nc >> 3;                     // channel groups (k-blocks) per timestep, <= KPT
-    const int tpb = KBB / kpt;                   // whole timesteps per batch
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
-
-    // slots q and q+4 of group 0 (channel offsets from the reference frequency) and the group step
-    const f2p dq = dup(float(a.frequencies[md.channel_begin + q] / kSpeedOfLight - s.f_ref));
-    const f2p dq4 = dup(float(a.frequencies[md.channel_begin + q + 4] / kSpeedOfLight - s.f_ref));
-    const f2p est = dup(8.0f * a.channel_step);
-
-    f2p pl[MT], pm[MT], pn[MT];
-    float acc[MT][4];
-#pragma unroll
-    for (int i = 0; i < MT; ++i) {
-        float l2[2], m2[2], n2[2];
-#pragma unroll
-        for (int r = 0; r < 2; ++r) {
-            const int pix = (warp * MT + i) * 16 + g + 8 * r;
-            const int x = pix % NS, y = pix / NS;
-            l2[r] = float(x - h) * a.cell_l;
-            m2[r] = float(y - h) * a.cell_l;
-            n2[r] = dev::w_term_n(l2[r], m2[r]);
-        }
-        pl[i] = pk(l2[0], l2[1]);
-        pm[i] = pk(m2[0], m2[1]);
-        pn[i] = pk(n2[0], n2[1]);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
-    }
-    float cur_scale = 0.0f;
-
-    const int64_t row = int64_t(a.nr_channels) * 4;  // float2 per timestep
-    const float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
-                         int64_t(md.channel_begin) * 4;
-
-    for (int t0 = 0; t0 < md.nr_timesteps; t0 += tpb) {
-        const int t1 = min(t0 + tpb, md.nr_timesteps);
-        const int nkb = (t1 - t0) * kpt;
-        const int nvb = nkb * 8;
-        __syncthreads();  // previous batch fully consumed
-        // (1) raw visibilities of timesteps [t0, t1): index j = (t - t0) nc + c
-        for (int i = threadIdx.x; i < 2 * nvb; i += NT) {
-            const int j = i >> 1;
-            const int t = j / nc, c = j - t * nc;
-            raw_s[i] = dev::ld_stream(reinterpret_cast<const float4 *>(vis0 + int64_t(t0 + t) * row + c * 4) + (i & 1));
-        }
-        // (2) per-timestep phase coefficients (fp64 -> fp32)
-        for (int t = t0 + int(threadIdx.x); t < t1; t += NT) {
-            float4 cB, cQ;
-            dev::timestep_coefficients(a, s, md.time_offset + t, cB, cQ);
-            coef_s[2 * (t - t0)] = cB;
-            coef_s[2 * (t - t0) + 1] = cQ;
-        }
-        __syncthreads();
-        // (3) f16 range: power-of-two scale from the batch maximum; never increase the running scale
-        float mx = 0.0f;
-        for (int i = threadIdx.x; i < 2 * nvb; i += NT) mx = abs_max4(raw_s[i], mx).x;
-        const float bscale = pow2_scale(block_max<WARPS>(mx, red_s));
-        if (cur_scale == 0.0f) {
-            cur_scale = bscale;
-        } else if (bscale < cur_scale) {
-            const float f = bscale / cur_scale;  // exact power of two
-#pragma unroll
-            for (int i = 0; i < MT; ++i)
-#pragma unroll
-                for (int j = 0; j < 4; ++j) acc[i][j] *= f;
-            cur_scale = bscale;
-        }
-        // (4) B fragments of every (timestep, group): column g = 2 pol + im, k-slots q and q+4
-        for (int i = threadIdx.x; i < nkb * 32; i += NT) {
-            const int kbl = i >> 5, ln = i & 31, gg = ln >> 2, qq = ln & 3;
-            const int pol = gg >> 1, im = gg & 1;
-            uint32_t hi[2], lo[2];
-#pragma unroll
-            for (int r = 0; r < 2; ++r) {
-                const float4 v4 = raw_s[2 * (kbl * 8 + qq + 4 * r) + (pol >> 1)];
-                const float vr = ((pol & 1) ? v4.z : v4.x) * cur_scale;
-                const float vi = ((pol & 1) ? v4.w : v4.y) * cur_scale;
-                split2(im ? vi : vr, im ? vr : -vi, hi[r], lo[r]);
-            }
-            frag_s[i] = make_uint4(hi[0], hi[1], lo[0], lo[1]);
-        }
-        __syncthreads();
-        // (5) per timestep: group-0 phasors of every tile, E_t, and one fresh D_j per group
-#pragma unroll 1
-        for (int t = t0; t < t1; ++t) {
-            const float4 cB = coef_s[2 * (t - t0)], cQ = coef_s[2 * (t - t0) + 1];
-            const uint4 *fr = frag_s + (t - t0) * kpt * 32 + lane;
-#pragma unroll
-            for (int i = 0; i < MT; ++i) {
-                const f2p Bv = fma2(dup(cB.x), pl[i], fma2(dup(cB.y), pm[i], mul2(dup(cB.z), pn[i])));
-                const f2p Qv = fma2(dup(cQ.x), pl[i], fma2(dup(cQ.y), pm[i], mul2(dup(cQ.z), pn[i])));
-                const float2 ph0 = unpk(fma2(dq, Qv, Bv));    // (row g, row g+8) at slot q
-                const float2 ph1 = unpk(fma2(dq4, Qv, Bv));   // (row g, row g+8) at slot q+4
-                float sn[4], cs[4];
-                __sincosf(ph0.x, &sn[0], &cs[0]);
-                __sincosf(ph0.y, &sn[1], &cs[1]);
-                __sincosf(ph1.x, &sn[2], &cs[2]);
-                __sincosf(ph1.y, &sn[3], &cs[3]);
-                uint32_t ah[4], al[4];
-#pragma unroll
-                for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[j], al[j]);
-                float er0 = 1.0f, ei0 = 0.0f, er1 = 1.0f, ei1 = 0.0f;  // E_t of rows g, g+8
-                if (KPT > 1 && kpt > 1) {
-                    const float2 e = unpk(mul2(est, Qv));
-                    __sincosf(e.x, &ei0, &er0);
-                    __sincosf(e.y, &ei1, &er1);
-                }
-                float pr0 = 1.0f, pi0 = 0.0f, pr1 = 1.0f, pi1 = 0.0f;  // E_t^j
-#pragma unroll
-                for (int j = 0; j < KPT; ++j) {
-                    if (j > 0 && j >= kpt) break;
-                    const uint4 bf = fr[j * 32];
-                    float d[4];
-                    mma16816_zero(d, ah[0], ah[1], ah[2], ah[3], bf.x, bf.y);
-                    mma16816(d, ah[0], ah[1], ah[2], ah[3], bf.z, bf.w);
-                    mma16816(d, al[0], al[1], al[2], al[3], bf.x, bf.y);
-                    if (j == 0) {
-#pragma unroll
-                        for (int k = 0; k < 4; ++k) acc[i][k] += d[k];
-                    } else {
-                        if (j == 1) {
-                            pr0 = er0; pi0 = ei0; pr1 = er1; pi1 = ei1;
-                        } else {
-                            const float a0 = fmaf(pr0, er0, -pi0 * ei0), b0 = fmaf(pr0, ei0, pi0 * er0);
-                            const float a1 = fmaf(pr1, er1, -pi1 * ei1), b1 = fmaf(pr1, ei1, pi1 * er1);
-                            pr0 = a0; pi0 = b0; pr1 = a1; pi1 = b1;
-                        }
-                        acc[i][0] = fmaf(pr0, d[0], fmaf(-pi0, d[1], acc[i][0]));
-                        acc[i][1] = fmaf(pr0, d[1], fmaf(pi0, d[0], acc[i][1]));
-                        acc[i][2] = fmaf(pr1, d[2], fmaf(-pi1, d[3], acc[i][2]));
-                        acc[i][3] = fmaf(pr1, d[3], fmaf(pi1, d[2], acc[i][3]));
-                    }
-                }
-            }
-        }
-    }
-
-    // ---- epilogue: D fragments -> sub_s[pol][pixel], then a3 + a4 + a5 ---------------------------
-    __syncthreads();
-    float2 *sub_s = reinterpret_cast<float2 *>(smem);
-    float2 *tmp_s = sub_s + 4 * NPIX;
-    const float inv = cur_scale > 0.0f ? 1.0f / cur_scale : 1.0f;
-#pragma unroll
-    for (int i = 0; i < MT; ++i) {
-        const int p0 = (warp * MT + i) * 16 + g;
-        sub_s[q * NPIX + p0] = make_float2(acc[i][0] * inv, acc[i][1] * inv);
-        sub_s[q * NPIX + p0 + 8] = make_float2(acc[i][2] * inv, acc[i][3] * inv);
-    }
-    __syncthreads();
-    gridder_epilogue_tc<NS, WARPS>(a, s, sub_s, tmp_s, reinterpret_cast<uint4 *>(tmp_s + 4 * NPIX), red_s);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -791,8 +576,11 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
         // (3) f16 range: power-of-two scale from the batch maximum; never increase the running scale
         float mx = 0.0f;
         for (int i = threadIdx.x; i < 2 * nvb; i += NT) mx = abs_max4(raw_s[i], mx).x;
-        const float bscale = pow2_scale(block_max<WARPS>(mx, red_s));
-        if (cur_scale == 0.0f) {
+        // (an all-zero batch, e.g. flagged data, leaves the scale alone: it carries no range information)
+        const float bmax = block_max<WARPS>(mx, red_s);
+        const float bscale = bmax > 0.0f ? pow2_scale(bmax) : 0.0f;
+        if (bscale == 0.0f) {
+        } else if (cur_scale == 0.0f) {
             cur_scale = bscale;
         } else if (bscale < cur_scale) {
             const float f = bscale / cur_scale;  // exact power of two
@@ -1022,39 +810,7 @@ __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const I
     return __frcp_rn(scale);
 }
 
-// sincos of two phases on the FMA pipe (packed f32x2), for kernels whose MUFU (XU) pipe is the binding
-// unit: quadrant reduction k = rint(x 2/pi) by the 1.5 2^23 rounding constant, y = x - k pi/2 in two
-// Cody-Waite steps (|y| <= pi/4), minimax polynomials of degree 7 / 8 on [-pi/4, pi/4] (Cephes sinf /
-// cosf coefficients, ~1 ulp), then the quadrant rotation by k mod 4 (the low bits of the rounded
-// value).  Abs. error ~1e-7 for |x| < 2^10, below the __sincosf (MUFU) error at the phases used here.
-// Measured (LOFAR degridder, B200): one of the thread's four slot pairs per k-block on the FMA pipe
-// 41.2 -> 47.2 ms, two -> 56.4 ms: the loop is bound by the whole instruction stream, not the MUFU alone.
-__device__ __forceinline__ void sincos_poly2(f2p x, float2 &sn, float2 &cs) {
-    const f2p magic = dup(12582912.0f);
-    const f2p t = fma2(x, dup(0.636619772367581f), magic);
-    const f2p k = sub2(t, magic);
-    f2p y = fma2(k, dup(-1.57079637050628662f), x);
-    y = fma2(k, dup(4.37113900018624e-8f), y);
-    const f2p y2 = mul2(y, y);
-    f2p ps = fma2(y2, dup(-1.9515295891e-4f), dup(8.3321608736e-3f));
-    ps = fma2(y2, ps, dup(-1.6666654611e-1f));
-    const f2p sy = fma2(mul2(y, y2), ps, y);
-    f2p pc = fma2(y2, dup(2.443315711809948e-5f), dup(-1.388731625493765e-3f));
-    pc = fma2(y2, pc, dup(4.166664568298827e-2f));
-    pc = fma2(y2, pc, dup(-0.5f));
-    const f2p cy = fma2(y2, pc, dup(1.0f));
-    const float2 tt = unpk(t), s2 = unpk(sy), c2 = unpk(cy);
-    auto fix = [](float tq, float s0, float c0, float &so, float &co) {
-        const uint32_t qd = __float_as_uint(tq);
-        const float a = (qd & 1) ? c0 : s0, b = (qd & 1) ? s0 : c0;
-        so = __uint_as_float(__float_as_uint(a) ^ ((qd << 30) & 0x80000000u));
-        co = __uint_as_float(__float_as_uint(b) ^ (((qd + 1) << 30) & 0x80000000u));
-    };
-    fix(tt.x, s2.x, c2.x, sn.x, cs.x);
-    fix(tt.y, s2.y, c2.y, sn.y, cs.y);
-}
-
-template <int NS, int WARPS, int MT, int MINB, int POLY = 0>
+template <int NS, int WARPS, int MT, int MINB>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int NKB = NPIX / 8;
@@ -1116,19 +872,11 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 #pragma unroll
             for (int i = 0; i < MT; ++i) {
                 // phases of (row, slot q) and (row, slot q+4) in one FFMA2 chain per row
-                const f2p p0v = fma2(cu[i][0], l2, fma2(cv[i][0], m2, mul2(cw[i][0], n2)));
-                const float2 p0 = unpk(p0v);
+                const float2 p0 = unpk(fma2(cu[i][0], l2, fma2(cv[i][0], m2, mul2(cw[i][0], n2))));
                 const float2 p1 = unpk(fma2(cu[i][1], l2, fma2(cv[i][1], m2, mul2(cw[i][1], n2))));
                 float sn[4], cs[4];
-                if (POLY > i) {
-                    // POLY of the MT row-g slot pairs on the FMA pipe (MUFU relief)
-                    float2 s2, c2;
-                    sincos_poly2(p0v, s2, c2);
-                    sn[0] = s2.x; cs[0] = c2.x; sn[2] = s2.y; cs[2] = c2.y;
-                } else {
-                    __sincosf(p0.x, &sn[0], &cs[0]);  // row g,   slot q
-                    __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
-                }
+                __sincosf(p0.x, &sn[0], &cs[0]);  // row g,   slot q
+                __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
                 __sincosf(p1.x, &sn[1], &cs[1]);  // row g+8, slot q
                 __sincosf(p1.y, &sn[3], &cs[3]);  // row g+8, slot q+4
 #pragma unroll
@@ -1156,121 +904,6 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 }
 
 // ------------------------------------------------------------------------------------------------
-// degridder_tc2: degridder_tc with the k-block loop split into subgrid rows y and the N~/8 k-blocks of a
-// row (unrolled).  A k-block is 8 pixels of one row, so m is constant over the row: the phase of a
-// (visibility, pixel) slot pair is  u l + (v m_y) + w n  with v m_y formed once per row and visibility,
-// the thread's l pairs (6 distinct values for N~ = 24) kept in registers, and only n read from shared
-// memory per k-block: 2 FFMA2 per row and k-block instead of 3, one LDS instead of two, and the loop
-// overhead spread over a row.
-// ------------------------------------------------------------------------------------------------
-template <int NS, int WARPS, int MT, int MINB>
-__global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc2_kernel(const KernelArgs a) {
-    constexpr int NPIX = NS * NS;
-    constexpr int NXB = NS / 8;   // k-blocks per subgrid row
-    constexpr int h = NS / 2;
-    static_assert(NS % 8 == 0, "k-blocks within a row");
-    extern __shared__ __align__(16) unsigned char smem[];
-    const DegridSmem<NS> sm(smem, a.max_timesteps_in_item);
-    const uint4 *frag_s = sm.frag_s;
-    const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
-    const float *df_s = sm.df_s;
-    __shared__ float red_s[WARPS];
-
-    const int item = a.order[blockIdx.x];
-    const ItemSetup s = dev::item_setup(a, item, NS);
-    const idg_metadata &md = s.md;
-    const int nc = s.nc;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
-    const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s);
-
-    f2p lq[NXB];   // l of the thread's slots q, q+4 in each k-block of a row
-#pragma unroll
-    for (int xb = 0; xb < NXB; ++xb)
-        lq[xb] = pk(float(8 * xb + q - h) * a.cell_l, float(8 * xb + q + 4 - h) * a.cell_l);
-
-    const int nvis = md.nr_timesteps * nc;
-    const int ntiles = (nvis + 15) >> 4;
-    const float rnc = __frcp_rn(float(nc));
-    const bool fdiv = nvis < (1 << 22);
-    auto tstep = [&](int v) { return fdiv ? __float2int_rz((float(v) + 0.5f) * rnc) : v / nc; };
-    const int64_t row = int64_t(a.nr_channels) * 4;
-    float2 *vis0 = a.vis + (int64_t(md.baseline) * a.nr_timesteps + md.time_offset) * row +
-                   int64_t(md.channel_begin) * 4;
-    for (int tile0 = warp * MT; tile0 < ntiles; tile0 += WARPS * MT) {
-        float cu[MT][2], cv[MT][2], cw[MT][2];   // per-visibility coefficients of rows g and g+8
-        float acc[MT][4];
-#pragma unroll
-        for (int i = 0; i < MT; ++i) {
-#pragma unroll
-            for (int r = 0; r < 2; ++r) {
-                const int v = (tile0 + i) * 16 + g + 8 * r;
-                float fu = 0.0f, fv = 0.0f, fw = 0.0f;
-                if (v < nvis) {
-                    const int t = tstep(v), c = v - t * nc;
-                    const float4 cB = bq_s[2 * t], cQ = bq_s[2 * t + 1];
-                    const float df = df_s[c];
-                    fu = fmaf(df, cQ.x, cB.x);
-                    fv = fmaf(df, cQ.y, cB.y);
-                    fw = fmaf(df, cQ.z, cB.z);
-                }
-                cu[i][r] = fu;
-                cv[i][r] = fv;
-                cw[i][r] = fw;
-            }
-#pragma unroll
-            for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
-        }
-#pragma unroll 1
-        for (int y = 0; y < NS; ++y) {
-            const float m = float(y - h) * a.cell_l;
-            f2p vm[MT][2];
-#pragma unroll
-            for (int i = 0; i < MT; ++i)
-#pragma unroll
-                for (int r = 0; r < 2; ++r) vm[i][r] = dup(cv[i][r] * m);
-#pragma unroll
-            for (int xb = 0; xb < NXB; ++xb) {
-                const int kb = y * NXB + xb;
-                const uint4 bf = frag_s[kb * 32 + lane];
-                const float4 *rec = lmn_s + (kb * 4 + q) * 2 + 1;
-                const float2 nn = *reinterpret_cast<const float2 *>(rec);
-                const f2p n2 = pk(nn.x, nn.y);
-                uint32_t ah[MT][4], al[MT][4];
-#pragma unroll
-                for (int i = 0; i < MT; ++i) {
-                    const float2 p0 = unpk(fma2(dup(cu[i][0]), lq[xb], fma2(dup(cw[i][0]), n2, vm[i][0])));
-                    const float2 p1 = unpk(fma2(dup(cu[i][1]), lq[xb], fma2(dup(cw[i][1]), n2, vm[i][1])));
-                    float sn[4], cs[4];
-                    __sincosf(p0.x, &sn[0], &cs[0]);  // row g,   slot q
-                    __sincosf(p1.x, &sn[1], &cs[1]);  // row g+8, slot q
-                    __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
-                    __sincosf(p1.y, &sn[3], &cs[3]);  // row g+8, slot q+4
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[i][j], al[i][j]);
-                }
-#pragma unroll
-                for (int i = 0; i < MT; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
-#pragma unroll
-                for (int i = 0; i < MT; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
-#pragma unroll
-                for (int i = 0; i < MT; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < MT; ++i) {
-#pragma unroll
-            for (int r = 0; r < 2; ++r) {
-                const int v = (tile0 + i) * 16 + g + 8 * r;
-                if (v < nvis) {
-                    const int t = tstep(v), c = v - t * nc;
-                    vis0[int64_t(t) * row + c * 4 + q] = make_float2(acc[i][2 * r] * inv, acc[i][2 * r + 1] * inv);
-                }
-            }
-        }
-    }
-}
-
-// ------------------------------------------------------------------------------------------------
 // Tensor-core degridder with phasor rotation across channel groups (uniform channels, C~ % 32 == 0).
 // A warp takes 32 channels of one timestep as two m-tiles, so each thread's four A rows are the
 // channels c0 + g + 8r (r = 0..3) of the same timestep.  With the phase linear in frequency,
@@ -1279,7 +912,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc2_kernel(const K
 // 1..3 by complex products (fp32, on the FMA pipe) before the operand split.  Exact in exact
 // arithmetic; the rounding is that of up to three extra complex products per phasor.
 // ------------------------------------------------------------------------------------------------
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int TFL = 0>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int NKB = NPIX / 8;
@@ -1371,49 +1004,21 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                 for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
             } else {
                 // R = 8, 16: each tile's three products issued as soon as its two rows are split
-                if constexpr (TFL) {
-                    // lo(A) B_hi as two tf32 m16n8k8 (slots q and q+4) on the fp32 residuals: no lo repacking.
-                    // B_hi as fp32: the lane's f16 pairs {B[2q][g], B[2q+1][g]} (cos / sin rows of slot q)
-                    // are exactly the tf32 B registers {(k = q, g), (k = q+4, g)} of the slot-q product.
-                    const float2 b0 = __half22float2(*reinterpret_cast<const __half2 *>(&bf.x));
-                    const float2 b4 = __half22float2(*reinterpret_cast<const __half2 *>(&bf.y));
 #pragma unroll
-                    for (int i = 0; i < NTL; ++i) {
-                        uint32_t ah[4];
-                        float lc[4], ls[4];
+                for (int i = 0; i < NTL; ++i) {
+                    uint32_t ah[4], al[4];
 #pragma unroll
-                        for (int h2 = 0; h2 < 2; ++h2) {
-                            if (i > 0 || h2 > 0) {
-                                const f2p Cn = fma2(C, EC, mul2(S, NES));
-                                S = fma2(C, ES, mul2(S, EC));
-                                C = Cn;
-                            }
-                            const float2 cc = unpk(C), ss = unpk(S);
-                            split_hi_res(cc.x, ss.x, ah[h2], lc[h2], ls[h2]);
-                            split_hi_res(cc.y, ss.y, ah[2 + h2], lc[2 + h2], ls[2 + h2]);
+                    for (int h2 = 0; h2 < 2; ++h2) {
+                        if (i > 0 || h2 > 0) {
+                            const f2p Cn = fma2(C, EC, mul2(S, NES));
+                            S = fma2(C, ES, mul2(S, EC));
+                            C = Cn;
                         }
-                        mma16816(acc[i], ah[0], ah[1], ah[2], ah[3], bf.x, bf.y);
-                        mma16816(acc[i], ah[0], ah[1], ah[2], ah[3], bf.z, bf.w);
-                        mma1688_tf32(acc[i], lc[0], lc[1], ls[0], ls[1], b0.x, b0.y);
-                        mma1688_tf32(acc[i], lc[2], lc[3], ls[2], ls[3], b4.x, b4.y);
+                        const float2 cc = unpk(C), ss = unpk(S);
+                        split_phasor(cc.x, ss.x, ah[h2], al[h2]);
+                        split_phasor(cc.y, ss.y, ah[2 + h2], al[2 + h2]);
                     }
-                } else {
-#pragma unroll
-                    for (int i = 0; i < NTL; ++i) {
-                        uint32_t ah[4], al[4];
-#pragma unroll
-                        for (int h2 = 0; h2 < 2; ++h2) {
-                            if (i > 0 || h2 > 0) {
-                                const f2p Cn = fma2(C, EC, mul2(S, NES));
-                                S = fma2(C, ES, mul2(S, EC));
-                                C = Cn;
-                            }
-                            const float2 cc = unpk(C), ss = unpk(S);
-                            split_phasor(cc.x, ss.x, ah[h2], al[h2]);
-                            split_phasor(cc.y, ss.y, ah[2 + h2], al[2 + h2]);
-                        }
-                        mma3(acc[i], ah, al, bf);
-                    }
+                    mma3(acc[i], ah, al, bf);
                 }
             }
         }
@@ -1472,183 +1077,109 @@ cudaError_t ensure_dft_tables() {
     }
     err = cudaMemcpyToSymbol(g_dft_tab, tab.data(), tab.size() * sizeof(uint4));
     if (err != cudaSuccess) return err;
+    // a pageable upload may return before its DMA has finished, and kernels launched on non-blocking
+    // streams are not ordered after it: wait for it once per device before any kernel reads the table
+    err = cudaDeviceSynchronize();
+    if (err != cudaSuccess) return err;
     if (done.size() <= size_t(dev)) done.resize(size_t(dev) + 1, 0);
     done[dev] = 1;
     return cudaSuccess;
 }
 
-template <int NS, int WARPS, int MT, int MINB, int REC, int KBB = kTcBatchKB>
+// ------------------------------------------------------------------------------------------------
+// Launchers and the variant tables.  Each variant names its dynamic shared memory (smem_*), so the
+// dispatcher can skip variants a plan's items do not fit (idg_kernels.cu: eligible()).
+// ------------------------------------------------------------------------------------------------
+template <typename K>
+cudaError_t launch_tc(K kernel, const char *name, size_t smem, int threads, const KernelArgs &a, cudaStream_t st) {
+    cudaError_t err = ensure_dft_tables();
+    if (err != cudaSuccess) return err;
+    if ((err = dev::prepare(kernel, smem)) != cudaSuccess) return err;
+    LaunchScope scope(name, st);
+    kernel<<<unsigned(a.nr_items), threads, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+template <int NS, int WARPS, int MT, int MINB, int KBB = kTcBatchKB>
+size_t smem_gridder_tc(const KernelArgs &a) { return gridder_tc_smem_bytes(NS, a.max_channels_in_item, KBB); }
+template <int NS, int WARPS, int MT, int MINB, int KBB = kTcBatchKB>
 cudaError_t launch_gridder_tc(const KernelArgs &a, cudaStream_t st) {
-    cudaError_t terr = ensure_dft_tables();
-    if (terr != cudaSuccess) return terr;
-    const size_t smem = gridder_tc_smem_bytes(NS, a.max_channels_in_item, KBB);
-    cudaError_t err = dev::prepare(gridder_tc_kernel<NS, WARPS, MT, MINB, REC, KBB>, smem);
-    if (err != cudaSuccess) return err;
-    LaunchScope scope("gridder", st);
-    gridder_tc_kernel<NS, WARPS, MT, MINB, REC, KBB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
-    return cudaGetLastError();
+    return launch_tc(gridder_tc_kernel<NS, WARPS, MT, MINB, KBB>, "gridder", smem_gridder_tc<NS, WARPS, MT, MINB, KBB>(a),
+                     WARPS * 32, a, st);
 }
 
-template <int NS, int WARPS, int MT, int MINB, int KPT, int KBB = kTcBatchKB>
-cudaError_t launch_gridder_rot(const KernelArgs &a, cudaStream_t st) {
-    cudaError_t terr = ensure_dft_tables();
-    if (terr != cudaSuccess) return terr;
-    const size_t smem = gridder_rot_smem_bytes(NS, KBB);
-    cudaError_t err = dev::prepare(gridder_rot_kernel<NS, WARPS, MT, MINB, KPT, KBB>, smem);
-    if (err != cudaSuccess) return err;
-    LaunchScope scope("gridder", st);
-    gridder_rot_kernel<NS, WARPS, MT, MINB, KPT, KBB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
-    return cudaGetLastError();
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int NSM = 0>
+size_t smem_gridder_rot2(const KernelArgs &) {
+    return gridder_rot_smem_bytes(NS, KBB) + size_t(NSM) * NS * NS * 4 + (NSM == 2 ? size_t(NS) * NS * 4 : 0);
 }
-
-template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int TU = 1, int NSM = 0>
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int NSM = 0>
 cudaError_t launch_gridder_rot2(const KernelArgs &a, cudaStream_t st) {
-    cudaError_t terr = ensure_dft_tables();
-    if (terr != cudaSuccess) return terr;
-    const size_t smem = gridder_rot_smem_bytes(NS, KBB) + size_t(NSM) * NS * NS * 4 + (NSM == 2 ? size_t(NS) * NS * 4 : 0);
-    cudaError_t err = dev::prepare(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, TU, NSM>, smem);
-    if (err != cudaSuccess) return err;
-    LaunchScope scope("gridder", st);
-    gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, TU, NSM><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
-    return cudaGetLastError();
+    return launch_tc(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, 1, NSM>, "gridder",
+                     smem_gridder_rot2<NS, WARPS, MT, MINB, KPT, GP, KBB, NSM>(a), WARPS * 32, a, st);
 }
 
-template <int NS, int WARPS, int MT, int MINB, int POLY = 0>
+template <int NS>
+size_t smem_degridder_tc(const KernelArgs &a) {
+    return degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
+}
+template <int NS, int WARPS, int MT, int MINB>
 cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
-    cudaError_t terr = ensure_dft_tables();
-    if (terr != cudaSuccess) return terr;
-    const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
-    cudaError_t err = dev::prepare(degridder_tc_kernel<NS, WARPS, MT, MINB, POLY>, smem);
-    if (err != cudaSuccess) return err;
-    LaunchScope scope("degridder", st);
-    degridder_tc_kernel<NS, WARPS, MT, MINB, POLY><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
-    return cudaGetLastError();
+    return launch_tc(degridder_tc_kernel<NS, WARPS, MT, MINB>, "degridder", smem_degridder_tc<NS>(a), WARPS * 32, a, st);
+}
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4>
+cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
+    return launch_tc(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R>, "degridder", smem_degridder_tc<NS>(a),
+                     WARPS * 32, a, st);
 }
 
-#define TGB(NS, W, MT, MB, KB) \
-    {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KB" #KB ">", launch_gridder_tc<NS, W, MT, MB, 0, KB>}
-#define TG(NS, W, MT, MB) \
-    {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB, 0>}
-#define TGR(NS, W, MT, MB) \
-    {NS, 8, kTensor, 1, "gridder_tcr<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB, 1>}
-// First eligible entry is the default.  B200 sweep (LOFAR, SKA-T1024): the direct kernel and the
-// channel-recurrence kernel run within 2% of each other (the kernels are latency-bound below the
-// XU limit), so the direct kernel (no recurrence error) is the default for N~ = 24; for N~ = 32 the
-// recurrence variant is 1% faster.
-#define TGROT(NS, W, MT, MB, KPT) \
-    {NS, 8, kTensor, 1, "gridder_rot<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ">", \
-     launch_gridder_rot<NS, W, MT, MB, KPT, 128>, 8 * KPT}
-// every item exactly 8 KPT channels (channel_gcd % 8 KPT == 0 and max channels <= 8 KPT)
+// Gridders.  First eligible entry is the default: the rotation gridder when every item has exactly 8 KPT
+// uniformly spaced channels (nsm / lmnsm: pixel coordinates re-read from shared memory, N~ = 32), else
+// the direct kernel (one sincos per pair; any channel table with C~ % 8 == 0), else the SIMT kernel.
 #define TGROT2(NS, W, MT, MB, KPT) \
     {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ">", \
-     launch_gridder_rot2<NS, W, MT, MB, KPT, KPT, 128>, 8 * KPT}
-#define TGROT2K(NS, W, MT, MB, KPT, KB) \
-    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",KB" #KB ">", \
-     launch_gridder_rot2<NS, W, MT, MB, KPT, KPT, KB>, 8 * KPT}
-#define TGROT2N(NS, W, MT, MB, KPT, GP) \
-    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP ",nsm>", \
-     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, 1, 1>, 8 * KPT}
-#define TGROT2N2(NS, W, MT, MB, KPT, GP) \
-    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP ",lmnsm>", \
-     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, 1, 2>, 8 * KPT}
-#define TGROT2P(NS, W, MT, MB, KPT, GP) \
-    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP ">", \
-     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128>, 8 * KPT}
+     launch_gridder_rot2<NS, W, MT, MB, KPT, KPT, 128>, 8 * KPT, smem_gridder_rot2<NS, W, MT, MB, KPT, KPT, 128>}
+#define TGROT2N(NS, W, MT, MB, KPT, GP, NSM, TAG) \
+    {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP "," TAG ">", \
+     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM>, 8 * KPT, smem_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM>}
+#define TG(NS, W, MT, MB) \
+    {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB>, 0, \
+     smem_gridder_tc<NS, W, MT, MB>}
 const Variant kTcGridder[] = {
     TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
-    TGROT2K(24, 12, 3, 2, 2, 64),
-    TGROT2N(32, 16, 4, 2, 4, 2), TGROT2N2(32, 16, 4, 2, 2, 2), TGROT2N(32, 16, 4, 2, 2, 2), TGROT2N2(24, 12, 3, 2, 2, 2), TGROT2P(32, 16, 4, 2, 4, 2), TGROT2(32, 16, 4, 1, 4), TGROT2P(32, 16, 4, 1, 4, 2), TGROT2P(32, 32, 2, 1, 4, 2), TGROT2(32, 32, 2, 1, 4), TGROT2(32, 16, 4, 2, 4), TGROT2(32, 16, 4, 2, 2), TGROT2(32, 16, 4, 1, 2), TGROT2(32, 32, 2, 1, 2), TGROT2(32, 16, 4, 2, 1),
+    TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
-    TGROT(24, 12, 3, 2, 4), TGROT(24, 12, 3, 2, 2), TGROT(24, 12, 3, 1, 2), TGROT(24, 12, 3, 1, 4),
-    TGROT(32, 16, 4, 2, 4), TGROT(32, 16, 4, 1, 4), TGROT(32, 16, 4, 1, 2), TGROT(32, 8, 8, 1, 4), TGROT(32, 16, 4, 1, 8),
-    TGROT(16, 8, 2, 2, 2), TGROT(16, 8, 2, 2, 4), TGROT(24, 12, 3, 1, 8),
-    TGROT(32, 32, 2, 1, 4), TGROT(24, 18, 2, 1, 4), TGROT(24, 18, 2, 1, 2),
-    TGB(24, 12, 3, 2, 128), TG(24, 12, 3, 2), TG(24, 6, 6, 2), TG(24, 9, 4, 2), TG(24, 4, 9, 3), TG(24, 18, 2, 1), TG(24, 12, 3, 1),
-    TG(24, 6, 6, 3), TG(24, 9, 4, 3), TG(24, 4, 9, 4),
-    TGR(32, 16, 4, 2), TGR(32, 8, 8, 2), TGR(32, 16, 4, 1),
-    TG(32, 16, 4, 2), TG(32, 8, 8, 2), TG(32, 16, 4, 1), TG(32, 4, 16, 3), TG(32, 8, 8, 3),
-    TG(16, 4, 4, 4), TG(16, 8, 2, 3), TG(16, 16, 1, 2),
-    TGR(24, 12, 3, 2), TGR(24, 9, 4, 3), TGR(24, 6, 6, 2), TGR(24, 4, 9, 4), TGR(24, 12, 3, 1),
-    TGR(16, 4, 4, 4), TGR(16, 8, 2, 3),
-    TGB(24, 12, 3, 2, 32), TGB(24, 12, 3, 2, 256), TGB(32, 16, 4, 2, 128), TGB(32, 16, 4, 2, 32),
+    TG(24, 12, 3, 2), TG(32, 16, 4, 2), TG(16, 4, 4, 4),
 };
-#undef TGB
-#undef TGR
-#undef TGROT
 #undef TGROT2
-#undef TGROT2P
 #undef TGROT2N
-#undef TGROT2N2
-#undef TGROT2K
 #undef TG
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int TFL = 0>
-cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
-    cudaError_t terr = ensure_dft_tables();
-    if (terr != cudaSuccess) return terr;
-    const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
-    cudaError_t err = dev::prepare(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R, TFL>, smem);
-    if (err != cudaSuccess) return err;
-    LaunchScope scope("degridder", st);
-    degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R, TFL><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
-    return cudaGetLastError();
-}
 
-// every item exactly CPT (4, 8 or 16) channels
-#define TDROTC(NS, W, MB, U, CPT) \
-    {NS, CPT, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
-     launch_degridder_rot<NS, W, MB, U, CPT>, CPT}
-// R = 8 channel rows per lane (4 m-tiles per unit), every item exactly CPT channels
-#define TDROT8(NS, W, MB, U, CPT) \
-    {NS, CPT, kTensor, 1, "degridder_rot8<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
-     launch_degridder_rot<NS, W, MB, U, CPT, 8>, CPT}
-#define TDROT16(NS, W, MB, U, CPT) \
-    {NS, CPT, kTensor, 1, "degridder_rot16<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
-     launch_degridder_rot<NS, W, MB, U, CPT, 16>, CPT}
-// R = 16 with the lo(A) B_hi product as tf32 mma on the fp32 residuals
-#define TDROT16T(NS, W, MB, U, CPT) \
-    {NS, CPT, kTensor, 1, "degridder_rot16t<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
-     launch_degridder_rot<NS, W, MB, U, CPT, 16, 1>, CPT}
+// Degridders.  Default: the phasor-rotation kernel for the item's channel layout (16 channel rows per lane
+// for 16- / 32-channel items, 8 for 8, 4 for 4 and for any multiple of 32), else the direct kernel, else
+// the SIMT kernel.
+#define TDROTC(NS, W, MB, U, CPT, R, TAG) \
+    {NS, CPT, kTensor, 1, TAG "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, R>, CPT, smem_degridder_tc<NS>}
 #define TDROT(NS, W, MB, U) \
-    {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>}
+    {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>, 0, \
+     smem_degridder_tc<NS>}
 #define TD(NS, W, MT, MB) \
-    {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>}
-template <int NS, int WARPS, int MT, int MINB>
-cudaError_t launch_degridder_tc2(const KernelArgs &a, cudaStream_t st) {
-    cudaError_t terr = ensure_dft_tables();
-    if (terr != cudaSuccess) return terr;
-    const size_t smem = degridder_tc_smem_bytes(NS, a.max_timesteps_in_item, a.max_channels_in_item);
-    cudaError_t err = dev::prepare(degridder_tc2_kernel<NS, WARPS, MT, MINB>, smem);
-    if (err != cudaSuccess) return err;
-    LaunchScope scope("degridder", st);
-    degridder_tc2_kernel<NS, WARPS, MT, MINB><<<unsigned(a.nr_items), WARPS * 32, smem, st>>>(a);
-    return cudaGetLastError();
-}
-#define TD2(NS, W, MT, MB) \
-    {NS, 0, kTensor, 0, "degridder_tc2<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc2<NS, W, MT, MB>}
-#define TDP(NS, W, MT, MB, P) \
-    {NS, 0, kTensor, 0, "degridder_tcp<" #NS ",W" #W ",MT" #MT ",minB" #MB ",P" #P ">", launch_degridder_tc<NS, W, MT, MB, P>}
+    {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>, 0, \
+     smem_degridder_tc<NS>}
 const Variant kTcDegridder[] = {
-    TDROT16(24, 4, 3, 4, 16), TDROT16(24, 4, 3, 2, 16), TDROT16(24, 4, 3, 1, 16), TDROT16(24, 8, 2, 1, 16), TDROT8(24, 8, 2, 1, 16), TDROT8(24, 8, 3, 1, 16),
-    TDROT16(32, 8, 2, 2, 32), TDROT16(32, 8, 2, 2, 16), TDROT16(32, 8, 2, 1, 32), TDROT16(32, 8, 2, 1, 16), TDROT16(32, 16, 1, 1, 32), TDROT16(16, 8, 2, 1, 16), TDROT16(16, 8, 2, 1, 32), TDROT8(32, 16, 2, 1, 16), TDROT8(32, 16, 2, 1, 32), TDROT8(24, 8, 2, 1, 8), TDROT8(32, 16, 2, 1, 8), TDROT8(16, 8, 2, 1, 8),
-    TDROT(32, 16, 2, 2), TDROT(32, 16, 1, 2), TDROT(32, 16, 2, 1), TDROT(32, 16, 1, 1), TDROT(32, 32, 1, 1), TDROT(32, 32, 1, 2), TDROT(32, 8, 2, 1),
-    TDROT(24, 8, 4, 1), TDROT(24, 8, 3, 1), TDROT(24, 8, 3, 2), TDROT(16, 8, 4, 1),
-    TDROTC(24, 8, 4, 1, 16), TDROTC(24, 8, 3, 1, 16), TDROTC(24, 16, 2, 1, 16), TDROTC(24, 8, 4, 1, 8), TDROTC(24, 8, 4, 1, 4),
-    TDROTC(32, 16, 2, 1, 16), TDROTC(32, 16, 1, 2, 16), TDROTC(32, 16, 2, 2, 16), TDROTC(32, 16, 2, 1, 8), TDROTC(32, 16, 2, 1, 4),
-    TDROTC(16, 8, 4, 1, 16), TDROTC(16, 8, 4, 1, 8), TDROTC(16, 8, 4, 1, 4),
-    TD2(24, 8, 2, 4), TD2(24, 8, 2, 3), TD2(24, 8, 4, 2), TD2(32, 8, 2, 4), TD2(16, 8, 2, 4),
-    TD(24, 8, 2, 4), TD(24, 8, 2, 3), TD(24, 8, 4, 2), TD(24, 4, 4, 4), TD(24, 8, 8, 1), TD(24, 16, 2, 1),
-    TD(24, 4, 2, 6), TDP(24, 8, 2, 4, 1), TDROT16T(24, 4, 3, 1, 16),
-    TD(32, 8, 4, 2), TD(32, 4, 4, 3), TD(32, 8, 8, 1), TD(32, 16, 2, 1),
-    TD(16, 8, 4, 2), TD(16, 4, 4, 4), TD(16, 8, 2, 3),
+    TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"),
+    TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
+    TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
+    TDROTC(24, 8, 2, 1, 8, 8, "degridder_rot8"), TDROTC(32, 16, 2, 1, 8, 8, "degridder_rot8"),
+    TDROTC(16, 8, 2, 1, 8, 8, "degridder_rot8"),
+    TDROT(32, 16, 2, 2), TDROT(24, 8, 4, 1), TDROT(16, 8, 4, 1),
+    TDROTC(24, 8, 4, 1, 4, 4, "degridder_rot"), TDROTC(32, 16, 2, 1, 4, 4, "degridder_rot"),
+    TDROTC(16, 8, 4, 1, 4, 4, "degridder_rot"),
+    TD(24, 8, 2, 4), TD(32, 8, 4, 2), TD(16, 8, 4, 2),
 };
-#undef TD
-#undef TDP
-#undef TD2
-#undef TDROT
 #undef TDROTC
-#undef TDROT8
-#undef TDROT16
-#undef TDROT16T
+#undef TDROT
+#undef TD
 
 }  // namespace
 

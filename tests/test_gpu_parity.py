@@ -56,36 +56,29 @@ def gpu_degrid(obs, grid_np_or_t, aterms, taper, plan=None):
 
 CASES = [
     ("tiny", {}, "identity", "ones"),
-    ("tiny", {}, "identity", "spheroidal"),
-    ("small_dde", {}, None, "spheroidal"),
+    ("tiny", {}, "identity", "asymmetric"),
+    ("small_dde", {}, None, "asymmetric"),
     ("small_dde", dict(C=7, C_block=3), None, "spheroidal"),          # ragged channel blocks
     ("small_dde", dict(C=12), None, "spheroidal"),                   # 12 channels: V=4 degridder
-    ("lofar", dict(T=640, nr_stations=5), None, "spheroidal"),       # N~=24, N=2048, 16 ch
+    ("small_dde", dict(C=8), None, "asymmetric"),                    # 8 channels: rot8 degridder
+    ("lofar", dict(T=640, nr_stations=5), None, "asymmetric"),       # N~=24, N=2048, 16 ch
     ("lofar_dde", dict(T=512, nr_stations=5), None, "spheroidal"),   # + random A-terms, w0
-    ("ska", dict(T=384, nr_stations=4), None, "spheroidal"),         # N~=32, N=8192, 32 ch
+    ("ska", dict(T=384, nr_stations=4), None, "asymmetric"),         # N~=32, N=8192, 32 ch
+    ("predict", dict(T=256, nr_stations=4), None, "asymmetric"),     # N~=32, 16 ch
     ("predict", dict(T=256, nr_stations=4, C=8), None, "spheroidal"),  # N~=32, 8 ch: one k-block/timestep
     ("small_dde", dict(C=24, C_block=8), None, "spheroidal"),       # 3 channel blocks of 8
-    ("small_dde", dict(w_planes=4), None, "spheroidal"),            # W-stacking (NEXT-1, R-21)
+    ("small_dde", dict(w_planes=4), None, "asymmetric"),            # W-stacking (NEXT-1, R-21)
     ("lofar_dde", dict(T=512, nr_stations=5, w_planes=3), None, "spheroidal"),
     ("small_dde", dict(C=64), None, "spheroidal"),                   # 2 blocks of 32 channels per timestep
-    ("small_dde", dict(C=40, C_block=24), None, "spheroidal"),      # 24 + 16 channels: rotation J = 3 and 2
+    ("small_dde", dict(C=40, C_block=24), None, "spheroidal"),      # 24 + 16 channels: mixed item widths
+    ("lofar", dict(T=256, nr_stations=5, channels="gap_jitter"), None, "asymmetric"),  # real channel table
 ]
 
 
 KINDS = {
-    "default": (None, None),                       # default tensor-core kernels (split-f16 mma)
-    "tc": ("tc", "tc"),                            # direct tensor-core kernels (no channel recurrence)
-    "rec": ("gridder_tcr<*", "degridder_tc<*"),    # split-f16 gridder with the channel recurrence
-    "rot": ("gridder_rot<*", "degridder_rot<*"),   # accumulator / phasor rotation over channel groups
-    "rot2": ("gridder_rot2<*", "degridder_rot<*"), # rotation with E_t derived from the slot phasors
-    "rot8": ("gridder_rot2<*", "degridder_rot8<*"), # degridder: 8 channel rows per lane (0.25 sincos/pair)
-    "rot16": ("gridder_rot2<*", "degridder_rot16<*"), # degridder: 16 channel rows per lane
-    "rot16t": ("gridder_rot2<*", "degridder_rot16t<*"), # + lo(A) B_hi as tf32 mma
-    "tc2": ("gridder_rot2<*", "degridder_tc2<*"), # degridder: row-split phase (m per row, l in registers)
-    "poly": ("gridder_rot2<*", "degridder_tcp<*"), # degridder with part of the sincos on the FMA pipe
-    "tf32": ("gridder_tf32*", "degridder_tf32*"),  # split-tf32 tensor-core kernels
-    "umma": ("gridder_umma*", "degridder_tc<*"),    # tcgen05 / TMEM gridder
-    "simt": ("simt", "simt"),                      # CUDA-core kernels (the paper's structure)
+    "default": (None, None),   # default: rotation kernels where the channel layout allows, else direct
+    "tc": ("tc", "tc"),        # direct tensor-core kernels (one sincos per pair, any channel table)
+    "simt": ("simt", "simt"),  # CUDA-core kernels (the paper's structure)
 }
 
 
@@ -183,31 +176,68 @@ def test_full_size_adjoint_and_sampled_items(name, kind):
     assert rel_rms(got, ref) <= TOL
 
 
-@pytest.mark.parametrize("name,kw,chunk", [("small_dde", {}, 60000), ("lofar", dict(T=640, nr_stations=6), 300000),
-                                           ("small_dde", dict(C=7, C_block=3), 40000),
-                                           ("small_dde", dict(w_planes=3), 60000)])
-def test_host_streamed_calls(name, kw, chunk, monkeypatch):
-    """idg_grid_host / idg_degrid_host (work groups through triple-buffered staging) give the
-    device-resident results: degridding bit-identical, gridding equal up to atomic summation order."""
+@pytest.mark.parametrize("name,kw,chunk,drop", [("small_dde", {}, 60000, False),
+                                                ("lofar", dict(T=640, nr_stations=6), 300000, False),
+                                                ("small_dde", dict(C=7, C_block=3), 40000, False),
+                                                ("small_dde", dict(w_planes=3), 60000, False),
+                                                ("small_dde", {}, 50000, True)])
+def test_host_streamed_calls(name, kw, chunk, drop, monkeypatch):
+    """idg_grid_host / idg_degrid_host (work groups through triple-buffered staging) against the
+    oracle, and against the device-resident calls (degridding bit-identical).  drop: long baselines fall
+    off the grid, so some work groups hold dropped runs (zeroed on the device) or no items at all."""
+    import dataclasses
     monkeypatch.setenv("IDG_HOST_CHUNK_BYTES", str(chunk))     # several work groups even at small sizes
     obs = idgsynth.make_observation(name, **kw)
-    vis, aterms, tap = _inputs(obs)
+    if drop:
+        obs = dataclasses.replace(obs, image_size=obs.image_size * 6)
+    vis, aterms, tap = _inputs(obs, None, "asymmetric")
+    items, dropped = oracle.plan(obs)
+    assert (dropped > 0) == drop
     plan = idg.Plan.from_observation(obs)
     ws = idg.workspace(plan)
     uvw, at, tp = _dev(obs.uvw), _dev(aterms), _dev(tap)
     vis_h = torch.from_numpy(vis).pin_memory()
-    g_dev = gpu_grid(obs, vis, aterms, tap, plan)
-    g_host = torch.zeros_like(g_dev)
+    g_host = torch.zeros(oracle.grid_shape(obs), dtype=torch.complex64, device="cuda")
     idg.grid_host(plan, vis_h, uvw, at, tp, g_host, ws)
     idg.grid_host(plan, vis_h, uvw, at, tp, g_host, ws)      # accumulates, buffers reused across calls
     torch.cuda.synchronize()
-    assert rel_rms(g_host.cpu().numpy(), 2 * g_dev.cpu().numpy()) < 1e-6
-    G = _dev(idgsynth.make_grid(obs))
-    v_dev = gpu_degrid(obs, G, aterms, tap, plan)
-    v_host = torch.full(v_dev.shape, complex(3, 3), dtype=torch.complex64).pin_memory()
-    idg.degrid_host(plan, G, uvw, at, tp, v_host, ws)
+    ref = 2 * oracle.grid(obs, items, vis, aterms, tap)
+    assert rel_rms(g_host.cpu().numpy(), ref) <= TOL
+    G = idgsynth.make_grid(obs)
+    refv = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, G, aterms, tap))
+    Gd = _dev(G)
+    v_host = torch.full((obs.nr_baselines, obs.nr_timesteps, obs.nr_channels, 4), complex(3, 3),
+                        dtype=torch.complex64).pin_memory()
+    idg.degrid_host(plan, Gd, uvw, at, tp, v_host, ws)
     torch.cuda.synchronize()
+    assert rel_rms(v_host.numpy(), refv) <= TOL
+    if drop:
+        assert np.all(v_host.numpy()[refv == 0] == 0)          # dropped -> exactly 0
+    v_dev = gpu_degrid(obs, G, aterms, tap, plan)
     assert torch.equal(v_host, v_dev.cpu())
+
+
+def test_host_streamed_upload_waits_for_the_callers_stream():
+    """A non-blocking device->host copy into vis_h queued on the caller's stream right before
+    idg_grid_host (no synchronize in between): the uploads must see the new host data."""
+    obs = idgsynth.make_observation("small_dde")
+    vis, aterms, tap = _inputs(obs, None, "asymmetric")
+    plan = idg.Plan.from_observation(obs)
+    ws = idg.workspace(plan)
+    uvw, at, tp = _dev(obs.uvw), _dev(aterms), _dev(tap)
+    items, _ = oracle.plan(obs)
+    ref = oracle.grid(obs, items, vis, aterms, tap)
+    s = torch.cuda.Stream()
+    vis_d = _dev(vis)
+    for _ in range(3):
+        vis_h = torch.zeros(vis.shape, dtype=torch.complex64).pin_memory()
+        g = torch.zeros(oracle.grid_shape(obs), dtype=torch.complex64, device="cuda")
+        with torch.cuda.stream(s):
+            torch.cuda._sleep(50_000_000)                    # keep the stream busy: the copy lands late
+            vis_h.copy_(vis_d, non_blocking=True)
+            idg.grid_host(plan, vis_h, uvw, at, tp, g, ws, stream=s)
+        s.synchronize()
+        assert rel_rms(g.cpu().numpy(), ref) <= TOL
 
 
 @pytest.mark.slow
@@ -251,6 +281,127 @@ def test_full_size_configs_sampled(name):
     torch.cuda.synchronize()
     lhs, rhs = _inner_t(DG, V), _inner_t(G, gV)
     assert abs(lhs - rhs) / abs(lhs) < 1e-4, (lhs, rhs)
+
+
+# ------------------------------------------------------------------------------------------------
+# the full-size uv regime: long baselines of the FULL observations (same L, N, channels), so the
+# subgrids sit near the grid edge (|u| L > 90 % of N/2) where fp32 phase formation is hardest
+# ------------------------------------------------------------------------------------------------
+_FULL = {}
+
+
+def _full_obs(name):
+    if name not in _FULL:
+        _FULL[name] = idgsynth.make_observation(name)
+    return _FULL[name]
+
+
+# (config, longest baselines, time window): windows where the longest tracks reach their extreme |u|
+FULL_L = [("lofar", 4, 0), ("ska", 3, 3072), ("predict", 3, 0)]
+
+
+def _full_l_subset(name, k, t0):
+    full = _full_obs(name)
+    obs = full.select(full.longest_baselines(k), nr_timesteps=1024, time_begin=t0)
+    assert obs.image_size == full.image_size
+    f = obs.frequencies.max() / idgsynth.SPEED_OF_LIGHT
+    reach = float(np.abs(obs.uvw[:, :, :2]).max()) * f * obs.image_size / (obs.grid_size / 2)
+    assert reach > 0.9, reach            # the subset exercises the outer grid
+    return obs
+
+
+def _window(items, n, N):
+    """Grid rows / columns [y0, y1) x [x0, x1) the items cover (the GPU grid is 0 elsewhere)."""
+    return (int(items["y"].min()), int(items["y"].max()) + n, int(items["x"].min()), int(items["x"].max()) + n)
+
+
+@pytest.mark.parametrize("name,k,t0", FULL_L)
+def test_grid_full_l_subset_matches_oracle(name, k, t0, kind):
+    obs = _full_l_subset(name, k, t0)
+    vis = idgsynth.make_visibilities(obs)
+    aterms = idgsynth.make_aterms(obs, "random")
+    tap = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
+    items, dropped = oracle.plan(obs)
+    assert dropped == 0
+    ref = oracle.grid(obs, items, vis, aterms, tap)
+    got = gpu_grid(obs, vis, aterms, tap)
+    y0, y1, x0, x1 = _window(items, obs.subgrid_size, obs.grid_size)
+    win = got[..., y0:y1, x0:x1]
+    assert abs(float(torch.linalg.vector_norm(got)) - float(torch.linalg.vector_norm(win))) <= 1e-6 * float(
+        torch.linalg.vector_norm(win))
+    err = rel_rms(win.cpu().numpy(), ref[..., y0:y1, x0:x1])
+    print(f"grid[{kind}] full-L {name}: {len(items)} items, rel rms {err:.3e}")
+    assert err <= TOL, err
+
+
+@pytest.mark.parametrize("name,k,t0", FULL_L)
+def test_degrid_full_l_subset_matches_oracle(name, k, t0, kind):
+    obs = _full_l_subset(name, k, t0)
+    aterms = idgsynth.make_aterms(obs, "random")
+    tap = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
+    items, _ = oracle.plan(obs)
+    y0, y1, x0, x1 = _window(items, obs.subgrid_size, obs.grid_size)
+    G = np.zeros(oracle.grid_shape(obs), dtype=np.complex64)       # random inside the covered window
+    rng = np.random.default_rng(obs.seed + 13)
+    shape = G[..., y0:y1, x0:x1].shape
+    G[..., y0:y1, x0:x1] = (rng.standard_normal(shape) + 1j * rng.standard_normal(shape)) * np.sqrt(0.5)
+    ref = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, G, aterms, tap))
+    got = gpu_degrid(obs, G, aterms, tap).cpu().numpy()
+    err = rel_rms(got, ref)
+    print(f"degrid[{kind}] full-L {name}: rel rms {err:.3e}")
+    assert err <= TOL, err
+
+
+def test_nonuniform_channels_use_direct_kernels():
+    """A real channel table (one channel missing, +-1 kHz jitter): the rotation kernels need uniformly
+    spaced channels, so the default dispatch must leave them, and the result still matches the oracle."""
+    full = _full_obs("lofar")
+    obs = idgsynth.make_observation("lofar", channels="gap_jitter").select(full.longest_baselines(3),
+                                                                          nr_timesteps=512)
+    assert np.ptp(np.diff(obs.frequencies)) > 1e3
+    vis = idgsynth.make_visibilities(obs)
+    aterms = idgsynth.make_aterms(obs, "random")
+    tap = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
+    items, _ = oracle.plan(obs)
+    ref = oracle.grid(obs, items, vis, aterms, tap)
+    got = gpu_grid(obs, vis, aterms, tap).cpu().numpy()
+    assert idg.last_variant("gridder").startswith("gridder_tc<"), idg.last_variant("gridder")
+    assert rel_rms(got, ref) <= TOL
+    G = idgsynth.make_grid(obs)
+    refv = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, G, aterms, tap))
+    gotv = gpu_degrid(obs, G, aterms, tap).cpu().numpy()
+    assert idg.last_variant("degridder").startswith("degridder_tc<"), idg.last_variant("degridder")
+    assert rel_rms(gotv, refv) <= TOL
+
+
+@pytest.mark.parametrize("name,kw", [("lofar", dict(T=640, nr_stations=5)), ("ska", dict(T=384, nr_stations=4))])
+def test_small_amplitudes_after_a_zero_batch(name, kw, kind):
+    """Visibilities of ~1e-4 (absolute units must not matter) whose first time steps are all zero (flagged):
+    the per-batch f16 range scale must not be pinned by the empty batch."""
+    obs = idgsynth.make_observation(name, **kw)
+    vis = idgsynth.make_visibilities(obs) * np.float32(1e-4)
+    vis[:, :200] = 0
+    aterms = idgsynth.make_aterms(obs, "random")
+    tap = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
+    items, _ = oracle.plan(obs)
+    ref = oracle.grid(obs, items, vis, aterms, tap)
+    err = rel_rms(gpu_grid(obs, vis, aterms, tap).cpu().numpy(), ref)
+    print(f"grid[{kind}] small amplitudes {name}: rel rms {err:.3e}")
+    assert err <= TOL, err
+
+
+def test_items_beyond_shared_memory_fall_back():
+    """Items of 8192 time steps: the tensor-core degridders stage per-timestep coefficients in shared
+    memory (32 B per step) and do not fit; the dispatcher must pick a kernel that does (not fail)."""
+    obs = idgsynth.make_observation("tiny", T=8192, dt=0.01, Tmax=8192, slot=8192)
+    items, _ = oracle.plan(obs)
+    assert int(items["nr_timesteps"].max()) > 7000
+    _, aterms, tap = _inputs(obs, "random", "asymmetric")
+    G = idgsynth.make_grid(obs)
+    ref = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, G, aterms, tap))
+    got = gpu_degrid(obs, G, aterms, tap).cpu().numpy()
+    assert idg.last_variant("degridder").startswith("degridder<"), idg.last_variant("degridder")
+    assert rel_rms(got, ref) <= TOL
 
 
 def test_tolerance_is_discriminating():

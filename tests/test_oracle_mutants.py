@@ -42,6 +42,10 @@ MUTANTS = [
      "or_mat_mul(tmp, Aq, res);\n            double s = 1.0;"),
     ("degridder taper skipped", "or_mat_mul(tmp, AqH, res);\n            double s = (double)taper[y * Ns + x];",
      "or_mat_mul(tmp, AqH, res);\n            double s = 1.0;"),
+    ("gridder taper transposed", "or_mat_mul(tmp, Aq, res);\n            double s = (double)taper[y * Ns + x];",
+     "or_mat_mul(tmp, Aq, res);\n            double s = (double)taper[x * Ns + y];"),
+    ("degridder taper transposed", "or_mat_mul(tmp, AqH, res);\n            double s = (double)taper[y * Ns + x];",
+     "or_mat_mul(tmp, AqH, res);\n            double s = (double)taper[x * Ns + y];"),
     ("adder one row low", "grid[(((int64_t)it->z * 4 + pol) * N + it->y + ky) * N + it->x + kx] +=",
      "grid[(((int64_t)it->z * 4 + pol) * N + it->y + ky + 1) * N + it->x + kx] +="),
     ("splitter transposed", "int64_t g = (((int64_t)it->z * 4 + pol) * N + it->y + ky) * N + it->x + kx;",

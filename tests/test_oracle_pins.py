@@ -96,7 +96,7 @@ def test_degrid_point_source_matches_eq1(pix):
     items, dropped = oracle.plan(obs)
     assert dropped == 0 and len(items) > 50
     items = items[::7]                                   # a spread of items keeps the test fast
-    taper = idgsynth.make_taper(obs.subgrid_size)
+    taper = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
     aterms = idgsynth.make_aterms(obs, "random")
     rng = np.random.default_rng(5)
     B = rng.standard_normal((2, 2)) + 1j * rng.standard_normal((2, 2))
@@ -113,7 +113,7 @@ def test_degrid_point_source_catches_w_sign():
     obs = idgsynth.make_observation("small_dde")
     items, _ = oracle.plan(obs)
     items = items[::11]
-    taper = idgsynth.make_taper(obs.subgrid_size)
+    taper = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
     aterms = idgsynth.make_aterms(obs, "random")
     B = np.array([[1.0, 0.3j], [-0.2, 0.7]])
     grid, (l0, m0, n0) = _point_source_case(obs, 12, 3, B, taper, aterms)
@@ -130,7 +130,7 @@ def test_adjoint_identity():
     obs = idgsynth.make_observation("small_dde")
     items, _ = oracle.plan(obs)
     items = items[::3]
-    taper = idgsynth.make_taper(obs.subgrid_size)
+    taper = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
     aterms = idgsynth.make_aterms(obs, "random")
     vis = idgsynth.make_visibilities(obs)
     G = idgsynth.make_grid(obs)
@@ -222,7 +222,7 @@ def test_w_stacking_point_source_matches_eq1_with_full_w_term():
     items, dropped = oracle.plan(obs)
     assert dropped == 0 and len(set(items["z"].tolist())) >= 3
     items = items[::5]
-    taper = idgsynth.make_taper(obs.subgrid_size)
+    taper = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
     aterms = idgsynth.make_aterms(obs, "random")
     B = np.array([[0.7 + 0.1j, -0.3j], [0.2, 1.1 - 0.4j]])
     x0, y0 = 10, 5
@@ -241,7 +241,7 @@ def test_w_stacking_adjoint_identity():
     obs = idgsynth.make_observation("small_dde", w_planes=3)
     items, _ = oracle.plan(obs)
     items = items[::3]
-    taper = idgsynth.make_taper(obs.subgrid_size)
+    taper = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
     aterms = idgsynth.make_aterms(obs, "random")
     vis = idgsynth.make_visibilities(obs)
     G = idgsynth.make_grid(obs)
