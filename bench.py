@@ -1,13 +1,15 @@
 #!/usr/bin/env python
 """IDG gridding + degridding throughput on B200 (BASELINE.json metric), one JSON line on rank 0.
 
-A step = one pass of the hot path over the LOFAR-shaped data set (BASELINE.json configs[1]):
+A step = one pass of the hot path over the SKA-low-shaped data set on an 8192^2 grid (BASELINE.json
+configs[3], the north star's 8-GPU target; --config lofar / lofar_dde / predict / tiny for the others):
     grid(visibilities) -> [N>1: NCCL reduce of the uv-grid to rank 0 -> broadcast] -> degrid(grid)
-The plan (host, built once per observation, "before any execution") is built before the timed
-region and reported separately as plan_s.  value = visibilities per step / step time (MVis/s),
-whole job; with N GPUs the baselines are split into N contiguous shards (strong scaling).
+(predict, configs[4]: broadcast of the model grid -> degrid only).  The plan (host, built once per
+observation, "before any execution") is built before the timed region and reported as plan_s.
+value = visibilities per step / step time (MVis/s), whole job; with N GPUs the baselines are split into
+N contiguous shards (strong scaling).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config lofar] [--impl ours|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config ska] [--impl ours|reference]
 
 --impl reference times the fp64 CPU oracle (oracle/, the correctness reference) on the host cores, on a
 bounded sample of the same workload per step; under torchrun only rank 0 runs it.
@@ -122,11 +124,10 @@ def workload_description(name):
 # ------------------------------------------------------------------------------------------------
 # CPU oracle (cpu_baseline / --impl reference)
 # ------------------------------------------------------------------------------------------------
-def oracle_sample(obs, target_s: float):
+def oracle_sample(obs, target_s: float, kind="grid+degrid"):
     """Choose a deterministic sample (first baselines x all timesteps) worth ~target_s of oracle time."""
-    import oracle
     probe = obs.subset(nr_baselines=1, nr_timesteps=min(obs.nr_timesteps, 16 * obs.max_timesteps_per_subgrid))
-    t = time_oracle_step(probe)[0]
+    t = time_oracle_step(probe, kind)[0]
     per_vis = t / max(1, probe.nr_visibilities)
     want_vis = target_s / max(per_vis, 1e-12)
     nt = obs.nr_timesteps
@@ -137,29 +138,34 @@ def oracle_sample(obs, target_s: float):
     return obs.subset(nr_baselines=nb, nr_timesteps=nt)
 
 
-def time_oracle_step(sample):
+def time_oracle_step(sample, kind="grid+degrid"):
     import oracle
     vis = idgsynth.make_visibilities(sample)
     aterms = idgsynth.make_aterms(sample)
     taper = idgsynth.make_taper(sample.subgrid_size)
     items, _ = oracle.plan(sample)
     t0 = time.perf_counter()
-    g = oracle.grid(sample, items, vis, aterms, taper)
+    if kind == "grid+degrid":
+        g = oracle.grid(sample, items, vis, aterms, taper).astype(np.complex64)
+    else:   # degrid only (predict): a model grid over the sample's covered window
+        g = np.zeros(oracle.grid_shape(sample), dtype=np.complex64)
+        g[..., items["y"].min():items["y"].max() + sample.subgrid_size,
+          items["x"].min():items["x"].max() + sample.subgrid_size] = 1.0
     t1 = time.perf_counter()
-    oracle.degrid(sample, items, g.astype(np.complex64), aterms, taper)
+    oracle.degrid(sample, items, g, aterms, taper)
     t2 = time.perf_counter()
     nvis = int(np.sum(items["nr_timesteps"].astype(np.int64) * (items["channel_end"] - items["channel_begin"])))
     return t2 - t0, nvis, t1 - t0, t2 - t1
 
 
-def cpu_baseline(obs, target_s=15.0):
+def cpu_baseline(obs, target_s=15.0, kind="grid+degrid"):
     import oracle
-    sample = oracle_sample(obs, target_s)
-    dt, nvis, tg, td = time_oracle_step(sample)
+    sample = oracle_sample(obs, target_s, kind)
+    dt, nvis, tg, td = time_oracle_step(sample, kind)
     return {"value": nvis / dt / 1e6, "unit": "MVis/s", "cores": oracle.max_threads(), "kind": "oracle",
             "sample": f"{sample.nr_baselines} baselines x {sample.nr_timesteps} timesteps x "
-                      f"{sample.nr_channels} channels of '{obs.name}' ({nvis} visibilities), grid {tg:.2f} s + "
-                      f"degrid {td:.2f} s, fp64 C + OpenMP"}
+                      f"{sample.nr_channels} channels of '{obs.name}' ({nvis} visibilities), step {kind}: grid "
+                      f"{tg:.2f} s + degrid {td:.2f} s, fp64 C + OpenMP"}
 
 
 def run_reference(args):
@@ -168,12 +174,13 @@ def run_reference(args):
         return 0
     import oracle
     obs = idgsynth.make_observation(args.config)
-    sample = oracle_sample(obs, args.reference_step_s)
+    kind = STEP_KIND[args.config]
+    sample = oracle_sample(obs, args.reference_step_s, kind)
     for _ in range(args.warmup):
-        time_oracle_step(sample)
+        time_oracle_step(sample, kind)
     times, nvis = [], 0
     for _ in range(args.steps):
-        dt, nvis, _, _ = time_oracle_step(sample)
+        dt, nvis, _, _ = time_oracle_step(sample, kind)
         times.append(dt)
     total = sum(times)
     value = nvis * args.steps / total / 1e6
@@ -181,7 +188,8 @@ def run_reference(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
-            "config": {"workload": workload_description(args.config), "sample_baselines": sample.nr_baselines,
+            "config": {"workload": workload_description(args.config), "step": kind,
+                       "sample_baselines": sample.nr_baselines,
                        "sample_timesteps": sample.nr_timesteps, "parallelism": "host OpenMP"},
             "cpu_baseline": {"value": value, "unit": "MVis/s", "cores": oracle.max_threads(), "kind": "oracle",
                              "sample": f"{sample.nr_baselines} baselines x {sample.nr_timesteps} timesteps x "
@@ -194,28 +202,78 @@ def run_reference(args):
 # ------------------------------------------------------------------------------------------------
 # our arm
 # ------------------------------------------------------------------------------------------------
+# A step per config: SKA-, LOFAR-shaped and tiny sets grid then degrid (the imaging cycle's two kernels,
+# P:45-47); the predict sweep (configs[4]) degrids only, from a model grid broadcast by rank 0.
+STEP_KIND = {"tiny": "grid+degrid", "lofar": "grid+degrid", "lofar_dde": "grid+degrid", "ska": "grid+degrid",
+             "predict": "degrid"}
+# e2e: the SKA-shaped set streams from the host as time chunks ("8 time chunks of 1024")
+E2E_TIME_CHUNK = {"ska": 1024}
+TENSOR_FLOPS_PER_PAIR = 96   # split-f16 contraction: 3 products x 16 real MACs x 2 flops per pair
+
+
 def sincos_per_pair(variant: str, nc_item: int) -> float:
-    """sincos evaluations per (pixel, visibility) pair of a kernel variant (the paper's kernels and
-    the direct tensor-core kernels: 1).  gridder_rot: per (pixel, timestep) 8 slot phasors + E_t in each
-    of the 4 lanes sharing the pixel, for 8 J pairs (J = channel groups of 8); gridder_rot2: the 8 slot
-    phasors only (E_t derived from slots q, q+4); gridder_tcr: half the
-    phasors by recurrence plus one step phasor per (pixel, timestep) in each of the 2 lanes;
-    degridder_rot / rot8 / rot16: per (visibility row 0, pixel) one phasor and one rotation E for 4 / 8 / 16
-    channel rows."""
+    """sincos evaluations per (pixel, visibility) pair of a kernel variant (the paper's kernels and the
+    direct tensor-core kernels: 1).  gridder_rot2: per (pixel, timestep) the 8 group-0 slot phasors for
+    8 J pairs (J = channel groups of 8; E_t is derived from them); degridder_rot / rot8 / rot16: per
+    (visibility row 0, pixel) one phasor and one rotation E for 4 / 8 / 16 channel rows."""
     j = max(1, nc_item // 8)
     if variant.startswith("gridder_rot2"):
-        return 1.0 / j  # the 8 group-0 phasors only; E_t is derived from them (no sincos)
+        return 1.0 / j
     if variant.startswith("gridder_rot"):
         return (8.0 + (4.0 if j > 1 else 0.0)) / (8.0 * j)
-    if variant.startswith("gridder_tcr"):
-        return 0.5 + 0.5 / j
     if variant.startswith("degridder_rot16"):
-        return 2.0 / 16  # per pixel slot: row 0 and E_tp for 16 channel rows
+        return 2.0 / 16
     if variant.startswith("degridder_rot8"):
         return 2.0 / 8
     if variant.startswith("degridder_rot"):
-        return 0.5     # per pixel slot: row 0 and E_tp for 4 channel rows
+        return 0.5
     return 1.0
+
+
+def sincos_fma_roofline(sm_mhz: float) -> float:
+    """The paper's sincos+FMA roofline of its formulation (17 FMA + 1 sincos per pair) from the
+    B200 unit counts: per SM and clock 128 FP32 FMA lanes (/17 per pair) and 16 MUFU lanes (/2 per sincos),
+    148 SMs, 36 paper-ops per pair; TOps/s at `sm_mhz`."""
+    return 148 * min(128.0 / 17.0, 16.0 / 2.0) * OPS_PER_PAIR * sm_mhz * 1e6 / 1e12
+
+
+def register_host(t):
+    """Page-lock an existing host tensor in place (cudaHostRegister: no power-of-two rounding of the
+    caching host allocator, which would turn a 94 GB buffer into 128 GB).  Returns True on success."""
+    import torch
+    try:
+        return int(torch._C._cudart.cudaHostRegister(t.data_ptr(), t.numel() * t.element_size(), 0)) == 0
+    except Exception:
+        return False
+
+
+def unregister_host(t):
+    import torch
+    try:
+        torch._C._cudart.cudaHostUnregister(t.data_ptr())
+    except Exception:
+        pass
+
+
+def host_buffer(shape, dtype):
+    """A page-locked host tensor (registered in place, else torch's pinned allocator)."""
+    import torch
+    t = torch.empty(shape, dtype=dtype)
+    if register_host(t):
+        return t, True
+    return torch.empty(shape, dtype=dtype, pin_memory=True), False
+
+
+def vdot_chunked(a, b, dev, chunk=1 << 27):
+    """sum conj(a) b in complex128 on the device, streaming host tensors through in chunks."""
+    import torch
+    a, b = a.reshape(-1), b.reshape(-1)
+    acc = torch.zeros((), dtype=torch.complex128, device=dev)
+    for i in range(0, a.numel(), chunk):
+        x = a[i:i + chunk].to(dev, non_blocking=True).to(torch.complex128)
+        y = b[i:i + chunk].to(dev, non_blocking=True).to(torch.complex128)
+        acc += torch.vdot(x, y)
+    return complex(acc.item())
 
 
 def run_ours(args):
@@ -240,6 +298,7 @@ def run_ours(args):
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=dev)
+    kind = STEP_KIND[args.config]
 
     over = {"T": args.timesteps} if args.timesteps else {}
     full = idgsynth.make_observation(args.config, **over)
@@ -251,29 +310,37 @@ def run_ours(args):
     st = plan.stats()
     pairs = st["nr_pairs"]
     nvis_rank = st["nr_vis_assigned"]
+    vis_shape = (obs.nr_baselines, obs.nr_timesteps, obs.nr_channels, 4)
+    vis_bytes = obs.nr_visibilities * 32
 
     aterms = idgsynth.make_aterms(obs)
     taper = idgsynth.make_taper(obs.subgrid_size)
     uvw_d = torch.from_numpy(obs.uvw).to(dev)
     at_d = torch.from_numpy(aterms).to(dev)
     tp_d = torch.from_numpy(taper).to(dev)
-    vis_d = idgsynth.torch_visibilities(obs, dev, seed_offset=11 + b0)
-    vis_bytes = vis_d.numel() * 8
-    free, _ = torch.cuda.mem_get_info(dev)
-    # the SKA-shaped set (94 GB) does not fit twice: degrid into the input buffer then (timing is
-    # value-independent; the next step grids the previous predictions)
-    inplace = free < vis_bytes + (16 << 30)
-    out_d = vis_d if inplace else torch.empty_like(vis_d)
     N = obs.grid_size
-    grid_d = torch.zeros((4, N, N), dtype=torch.complex64, device=dev)
     stream = torch.cuda.current_stream(dev)
-
     sharded = parallel.ShardedIDG(plan)
+    if kind == "grid+degrid":
+        vis_d = idgsynth.torch_visibilities(obs, dev, seed_offset=11 + b0)
+        free, _ = torch.cuda.mem_get_info(dev)
+        # the SKA-shaped set (94 GB) does not fit twice: degrid into the input buffer then (timing is
+        # value-independent; the next step grids the previous predictions)
+        inplace = free < vis_bytes + (16 << 30)
+        out_d = vis_d if inplace else torch.empty_like(vis_d)
+        grid_d = torch.zeros((4, N, N), dtype=torch.complex64, device=dev)
+    else:
+        # predict: degrid only; rank 0 holds the model grid (synthetic: values do not affect run time)
+        vis_d, inplace = None, False
+        out_d = torch.empty(vis_shape, dtype=torch.complex64, device=dev)
+        grid_d = idgsynth.torch_grid(obs, dev) if rank == 0 else torch.zeros((4, N, N), dtype=torch.complex64,
+                                                                             device=dev)
 
-    def step(vis_in, vis_out):
-        grid_d.zero_()
-        sharded.grid(vis_in, uvw_d, at_d, tp_d, grid_d, dst=0)       # + NCCL reduce of the uv-grids
-        sharded.degrid(grid_d, uvw_d, at_d, tp_d, vis_out, src=0)    # NCCL broadcast of the model grid
+    def step():
+        if kind == "grid+degrid":
+            grid_d.zero_()
+            sharded.grid(vis_d, uvw_d, at_d, tp_d, grid_d, dst=0)        # + NCCL reduce of the uv-grids
+        sharded.degrid(grid_d, uvw_d, at_d, tp_d, out_d, src=0)          # NCCL broadcast of the model grid
 
     def barrier():
         if world > 1:
@@ -281,7 +348,7 @@ def run_ours(args):
         torch.cuda.synchronize(dev)
 
     for _ in range(args.warmup):
-        step(vis_d, out_d)
+        step()
     barrier()
 
     # ---- timed region: device-resident inputs -------------------------------------------------
@@ -294,7 +361,7 @@ def run_ours(args):
         mj0 = clocks.energy_mj()
         ev0.record(stream)
         for _ in range(args.steps):
-            step(vis_d, out_d)
+            step()
         ev1.record(stream)
         barrier()
         mj1 = clocks.energy_mj()
@@ -311,113 +378,68 @@ def run_ours(args):
         dist.all_reduce(nvis_t)
     nvis_total = float(nvis_t.item())
     value = nvis_total * args.steps / (ms_max * 1e-3) / 1e6
-    # energy efficiency (Fig. 15: GFlops/W per kernel; here the whole step, board energy)
+    md = plan.metadata()
+    nc_item = int((md["channel_end"] - md["channel_begin"]).max()) if len(md) else 1
+    kernels_in_step = ["gridder", "degridder"] if kind == "grid+degrid" else ["degridder"]
     energy = None
     if mj0 is not None and mj1 is not None and mj1 > mj0:
         joules = (mj1 - mj0) / 1e3
-        ops = 2 * OPS_PER_PAIR * float(pairs) * args.steps       # grid + degrid pairs on this rank
+        ops = len(kernels_in_step) * OPS_PER_PAIR * float(pairs) * args.steps
         energy = {"J_per_step": joules / args.steps, "avg_W": joules / (ms * 1e-3),
-                  "GOps_per_J": ops / joules / 1e9, "source": "NVML total energy counter, this GPU, timed region",
-                  "paper_context": "GTX 1080: 32 / 23 GFlops/W gridder / degridder (P:306)"}
+                  "GOps_per_J": ops / joules / 1e9, "source": "NVML total energy counter, this GPU, timed region"}
+
+    # ---- energy per kernel (Fig. 15: GFlops/W of the gridder and the degridder) -----------
+    # separate timed loops of one kernel each, NVML board energy over the loop
+    if energy is not None and not args.no_kernel_energy:
+        per = {}
+        n_e = max(3, min(args.steps, args.energy_launches))
+        loops = {"gridder": lambda: idg.grid(plan, vis_d, uvw_d, at_d, tp_d, grid_d),
+                 "degridder": lambda: idg.degrid(plan, grid_d, uvw_d, at_d, tp_d, out_d)}
+        for name in kernels_in_step:
+            barrier()
+            if name == "gridder":
+                grid_d.zero_()
+            e_a, e_b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            barrier()
+            mja = clocks.energy_mj()
+            e_a.record(stream)
+            for _ in range(n_e):
+                loops[name]()
+            e_b.record(stream)
+            barrier()
+            mjb = clocks.energy_mj()
+            if mja is None or mjb is None or mjb <= mja:
+                continue
+            J = (mjb - mja) / 1e3 / n_e
+            sec = e_a.elapsed_time(e_b) * 1e-3 / n_e
+            spp = sincos_per_pair(idg.last_variant(name), nc_item)
+            per[name] = {"launches": n_e, "J_per_launch": J, "s_per_launch": sec, "avg_W": J / sec,
+                         "paper_GOps_per_J": OPS_PER_PAIR * pairs / J / 1e9,
+                         "executed_tensor_GFlops_per_J": TENSOR_FLOPS_PER_PAIR * pairs / J / 1e9,
+                         "executed_sincos_G_per_J": spp * pairs / J / 1e9,
+                         "executed": f"per pair: {TENSOR_FLOPS_PER_PAIR} tensor-core flops (3 split-f16 products), "
+                                     f"{spp:g} sincos (MUFU), phasor rotation + operand split on the ALUs"}
+        energy["per_kernel"] = per
+        energy["paper_context"] = "GTX 1080: 32 / 23 GFlops/W gridder / degridder (P:306; paper-ops: 17 FMA + sincos)"
 
     # ---- e2e: host buffers through the public API ------------------------------------------------
-    # Every step uploads its inputs (visibilities, uvw) from pinned host memory and downloads the
-    # predicted visibilities: idg_grid_host / idg_degrid_host stream the visibilities in work groups
-    # through triple-buffered staging buffers so the PCIe transfers overlap the kernels.
-    e2e = None
-    try:
-        import psutil
-        host_avail = psutil.virtual_memory().available
-    except Exception:
-        host_avail = None
-    e2e_fits = host_avail is None or 3 * vis_bytes < 0.7 * host_avail
-    free, _ = torch.cuda.mem_get_info(dev)
-    e2e_fits = e2e_fits and (inplace or free + vis_bytes > 2.2 * vis_bytes)
-    if not args.no_e2e and not e2e_fits:
-        e2e = {"value": None, "unit": "MVis/s", "skipped": "pinned host buffers for the inputs and outputs "
-               f"({2 * vis_bytes / 1e9:.0f} GB) do not fit this host/device"}
-    if not args.no_e2e and e2e_fits:
-        vis_h = torch.empty(vis_d.shape, dtype=vis_d.dtype, pin_memory=True)
-        vis_h.copy_(vis_d)
-        out_hs = [torch.empty_like(vis_h, pin_memory=True) for _ in range(2)]
-        uvw_h = torch.from_numpy(obs.uvw).pin_memory()
-        # reference for the e2e result: the device-resident path's predictions of a few baselines
-        # (same inputs; they differ only by the grid's atomic summation order)
-        nb_chk = min(16, obs.nr_baselines)
-        if not inplace:
-            step(vis_d, out_d)
-            chk_ref = out_d[:nb_chk].cpu()
-        else:
-            chk_ref = None
-        del vis_d, out_d
-        torch.cuda.empty_cache()
-        # one workspace and one output buffer per stream: a workspace serves one in-flight call
-        wss = [idg.workspace(plan, dev, full=True) for _ in range(2)]
-
-        # Independent steps alternate between two streams (and two grids): each call is complete on
-        # its own stream (idg_degrid_host's downloads included), while step k+1's uploads and gridding
-        # overlap step k's degridding and downloads.
-        streams = [stream, torch.cuda.Stream(dev)]
-        grids = [grid_d, torch.zeros_like(grid_d)]
-        uvws = [uvw_d, torch.empty_like(uvw_d)]
-
-        def e2e_step(k):
-            s_k, g_k, u_k, w_k, o_k = streams[k % 2], grids[k % 2], uvws[k % 2], wss[k % 2], out_hs[k % 2]
-            with torch.cuda.stream(s_k):
-                u_k.copy_(uvw_h, non_blocking=True)
-                g_k.zero_()
-                sharded.grid_host(vis_h, u_k, at_d, tp_d, g_k, w_k, dst=0, stream=s_k)
-                sharded.degrid_host(g_k, u_k, at_d, tp_d, o_k, w_k, src=0, stream=s_k)
-
-        e2e_step(0)
-        e2e_step(1)
-        barrier()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        ksteps = max(1, min(args.steps, args.e2e_steps))
-        e0.record(stream)
-        streams[1].wait_event(e0)
-        for k in range(ksteps):
-            e2e_step(k)
-        last = torch.cuda.Event()
-        last.record(streams[1])
-        stream.wait_event(last)
-        e1.record(stream)
-        barrier()
-        te = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        chk = None
-        if chk_ref is not None:
-            got = out_hs[(ksteps - 1) % 2][:nb_chk]
-            chk = float(torch.linalg.vector_norm(got - chk_ref) / torch.linalg.vector_norm(chk_ref))
-        e2e = {"value": nvis_total * ksteps / (float(te.item()) * 1e-3) / 1e6, "unit": "MVis/s",
-               "h2d_bytes_per_step": int(vis_h.numel() * 8 + uvw_h.numel() * 4),
-               "d2h_bytes_per_step": int(out_hs[0].numel() * 8), "steps": ksteps,
-               "check_rel_rms_vs_device_path": chk,
-               "api": "idg_grid_host + idg_degrid_host (host-streamed work groups, one staging buffer per "
-                      "work group; independent steps on two alternating streams so the uploads of step k+1 "
-                      "overlap the degridding and downloads of step k)"}
-        del vis_h, out_hs, wss
+    e2e = None if args.no_e2e else run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream,
+                                           world, rank, nvis_total, vis_d, out_d, grid_d, sharded, barrier, inplace)
+    del vis_d, out_d
 
     # ---- roofline ---------------------------------------------------------------------------------
-    # The tensor-core kernels run the 16 multiply-adds per pair on the tensor cores; what bounds them
-    # is the sincos rate of the XU (MUFU) pipe: one sincos per (pixel, visibility) pair.  Its measured
-    # throughput (rho = 0 benchmark) x 36 paper-ops is the roofline; the paper's own modified roofline
-    # (FMA:sincos mix at rho = 17) is reported beside it.  Best of 3, same process, clocks
-    # sampled while they run.
-    def best(rho, iters):
-        return max(idg.rho_benchmark(rho, iters)[0] for _ in range(3))
+    def best(rho, iters, scalar=False):
+        return max(idg.rho_benchmark(rho, iters, scalar=scalar)[0] for _ in range(3))
     with ClockSampler(local) as rclocks:
         sincos_per_s = best(0, 4 * args.rho_iterations) / 2.0
         rho17 = best(17, args.rho_iterations) / 1e12
+        rho17_scalar = best(17, args.rho_iterations, scalar=True) / 1e12
+        rho_sweep = {}
+        if not args.no_rho_sweep:
+            for r in (0, 1, 2, 4, 8, 12, 16, 17, 24, 32, 64):
+                rho_sweep[str(r)] = best(r, args.rho_iterations) / 1e12
     xu_peak = sincos_per_s * OPS_PER_PAIR / 1e12
-    rho_sweep = {}
-    if args.rho_sweep:
-        for r in (0, 1, 2, 4, 8, 12, 16, 17, 24, 32, 64):
-            rho_sweep[str(r)] = best(r, args.rho_iterations) / 1e12
     per_kernel = {}
-    md = plan.metadata()
-    nc_item = int((md["channel_end"] - md["channel_begin"]).max()) if len(md) else 1
     for name in ("gridder", "degridder"):
         k = kern.get(name)
         if not k:
@@ -427,46 +449,40 @@ def run_ours(args):
         variant = idg.last_variant(name)
         spp = sincos_per_pair(variant, nc_item)
         per_kernel[name] = {"launches": k["launches"], "avg_ms": avg_ms, "TOps_s": achieved,
-                            "frac_xu_sincos": achieved / xu_peak, "frac_rho17": achieved / rho17,
-                            "share_of_step": k["total_ms"] / ms, "variant": variant,
-                            "sincos_per_pair": spp, "peak_own_TOps_s": xu_peak / spp,
-                            "frac_own_bound": achieved * spp / xu_peak}
+                            "mvis_s": nvis_rank / (avg_ms * 1e-3) / 1e6,
+                            "frac_rho17": achieved / rho17, "share_of_step": k["total_ms"] / ms, "variant": variant,
+                            "sincos_per_pair": spp, "peak_own_xu_TOps_s": xu_peak / spp,
+                            "frac_own_xu_bound": achieved * spp / xu_peak}
     dominant = max(per_kernel, key=lambda n: per_kernel[n]["avg_ms"]) if per_kernel else None
     sm_mhz = clocks.summary()["sm_mhz"] or 1965
-    traffic = None
+    hw = None
     prof_json = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if dominant and os.path.exists(prof_json):
         try:
-            traffic = json.load(open(prof_json)).get(args.config, {}).get(dominant, {}).get("dram_bytes")
+            hw = json.load(open(prof_json)).get(args.config, {}).get(dominant)
         except Exception:
-            traffic = None
-    # peak: the one-sincos-per-pair roofline from the unit counts at the clock of the timed region
-    # (148 SMs x 16 MUFU lanes/clk / 2 MUFU per sincos x 36 paper-ops per pair).  It is a hard ceiling for
-    # the paper's formulation (one sincos per pair); the rotation kernels evaluate fewer
-    # sincos, so for them it is the paper-metric ceiling, and their own sincos bound is reported per kernel.
-    xu_theory = 148 * 8 * OPS_PER_PAIR * sm_mhz * 1e6 / 1e12
+            hw = None
+    peak = sincos_fma_roofline(sm_mhz)
     for k in per_kernel.values():
-        k["frac_xu_theoretical"] = k["TOps_s"] / xu_theory
+        k["frac_sincos_fma_roofline"] = k["TOps_s"] / peak
     roofline = None
     if dominant:
         roofline = {"bound": "alu", "kernel": dominant, "achieved": per_kernel[dominant]["TOps_s"],
-                    "peak": xu_theory, "unit": "TOps/s", "frac": per_kernel[dominant]["TOps_s"] / xu_theory,
-                    "traffic": traffic,
-                    "peak_source": "one-sincos-per-pair roofline from unit counts at the timed region's SM clock: "
-                                   "148 SMs x 16 MUFU lanes/clk / 2 (sin + cos) x 36 paper-ops per pair "
-                                   "(P:258, P:276); the paper's formulation cannot exceed it.  The B200 kernels "
-                                   "evaluate 0.125-0.5 sincos per pair (rotation), so their own sincos bound "
-                                   "(kernels[*].peak_own_TOps_s) is higher; what binds them is instruction issue "
-                                   "(see DESIGN.md section 7)",
-                    "peak_measured_xu": xu_peak, "frac_measured_xu": per_kernel[dominant]["frac_xu_sincos"],
-                    "peak_measured_xu_source": "measured sincos throughput of the XU/MUFU pipe "
-                                               "(idg_rho_benchmark rho=0, best of 3) x 36, this process",
+                    "peak": peak, "unit": "TOps/s", "frac": per_kernel[dominant]["TOps_s"] / peak,
+                    "traffic": (hw or {}).get("dram_bytes"),
+                    "peak_source": "the paper's sincos+FMA roofline (P:276-290) from B200 unit counts at the timed "
+                                   "region's SM clock: 148 SMs x min(128 FMA lanes / 17, 16 MUFU lanes / 2) pairs/clk "
+                                   "x 36 paper-ops per pair (P:258); a ceiling for the paper's formulation (17 FMA + "
+                                   "1 sincos per pair), which the B200 kernels leave (tensor-core MACs, sincos by "
+                                   "rotation): their hardware bound is roofline.hw",
                     "variant": per_kernel[dominant]["variant"],
-                    "peak_rho17": rho17, "frac_rho17": per_kernel[dominant]["frac_rho17"],
-                    "peak_rho17_source": "paper's modified roofline: FMA:sincos mix at rho=17 (P:276-290), "
-                                         "measured in this process",
+                    "peak_measured_rho17": rho17, "frac_measured_rho17": per_kernel[dominant]["TOps_s"] / rho17,
+                    "peak_measured_rho17_source": "paper's FMA:sincos benchmark at rho=17 (P:276-290), FMAs as packed "
+                                                  "FFMA2, measured in this process (best of 3)",
+                    "rho17_scalar_ffma": rho17_scalar,
+                    "peak_measured_xu": xu_peak,
                     "ops_per_pair": OPS_PER_PAIR, "pairs_per_launch": pairs,
-                    "clocks_during_peak": rclocks.summary()}
+                    "hw": hw, "clocks_during_peak": rclocks.summary()}
 
     if rank != 0:
         if world > 1:
@@ -474,23 +490,24 @@ def run_ours(args):
         return 0
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(full, args.cpu_baseline_s)
+        cpu = cpu_baseline(full, args.cpu_baseline_s, kind)
     line = {
         "metric": METRIC, "value": value, "unit": "MVis/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": workload_description(args.config) + (f" [T reduced to {args.timesteps}]" if args.timesteps else ""),
+                   "step": kind + (" (model grid broadcast from rank 0)" if kind == "degrid" else ""),
                    "visibilities": int(nvis_total),
                    "arithmetic": "fp32 phases + MUFU sincos; pixel x visibility products and the subgrid "
                                  "DFTs on tensor cores as split-f16 (hi*hi + hi*lo + lo*hi) mma with fp32 "
-                                 "accumulation; gridder: phasors of 8 channels per timestep rotated to the "
-                                 "other channel groups on the fp32 accumulators (uniform channels)",
+                                 "accumulation; sincos of one channel group / row per pixel, the other channels by "
+                                 "exact rotation (uniform channels)",
                    "subgrids_rank0": st["nr_subgrids"], "pairs_rank0": pairs,
                    "parallelism": f"baseline shards x{world}" + (" + NCCL reduce/broadcast" if world > 1 else ""),
                    "l2": f"inputs larger than L2 (visibilities {vis_bytes / 1e9:.1f} GB/step)",
                    "degrid_in_place": inplace},
-        "grid_mvis_s": (nvis_rank / (per_kernel["gridder"]["avg_ms"] * 1e-3) / 1e6) if "gridder" in per_kernel else None,
-        "degrid_mvis_s": (nvis_rank / (per_kernel["degridder"]["avg_ms"] * 1e-3) / 1e6) if "degridder" in per_kernel else None,
+        "grid_mvis_s": per_kernel.get("gridder", {}).get("mvis_s"),
+        "degrid_mvis_s": per_kernel.get("degridder", {}).get("mvis_s"),
         "plan_s": plan_s, "clocks": clocks.summary(), "energy": energy, "e2e": e2e, "gpu_launches": gpu_launches,
         "roofline": roofline, "kernels": per_kernel, "rho_sweep_TOps_s": rho_sweep or None,
         "cpu_baseline": cpu,
@@ -501,20 +518,170 @@ def run_ours(args):
     return 0
 
 
+def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, world, rank, nvis_total, vis_d,
+            out_d, grid_d, sharded, barrier, inplace):
+    """The metric end to end through the public host-streamed calls (idg_grid_host / idg_degrid_host, the
+    paper's triple-buffered work groups): every step uploads its inputs (visibilities, uvw,
+    A-terms; the model grid for predict) from page-locked host memory and downloads the predictions.
+    The SKA-shaped set streams as time chunks of 1024 (one plan per chunk)."""
+    import torch
+    import torch.distributed as dist
+    try:
+        import psutil
+        host_avail = psutil.virtual_memory().available
+    except Exception:
+        host_avail = None
+    T = obs.nr_timesteps
+    chunk_T = min(T, E2E_TIME_CHUNK.get(args.config, T))
+    nchunks = (T + chunk_T - 1) // chunk_T
+    nbl, C = obs.nr_baselines, obs.nr_channels
+    chunk_bytes = nbl * chunk_T * C * 32
+    vis_bytes = nbl * T * C * 32
+    n_in = 1 if kind == "grid+degrid" else 0
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", world))
+    # host memory of ALL local ranks: inputs + outputs (full arrays; the two in-flight steps download into
+    # the same host arrays), else 2 rotating chunk buffers per direction
+    need_full = local_world * (n_in + 1) * vis_bytes
+    need_rot = local_world * (n_in + 1) * 2 * chunk_bytes
+    if host_avail is not None and need_full > 0.7 * host_avail:
+        if nchunks == 1 or need_rot > 0.7 * host_avail:
+            return {"value": None, "unit": "MVis/s", "skipped": f"page-locked host buffers ({need_full / 1e9:.0f} GB for "
+                    f"{local_world} local ranks) do not fit the host ({host_avail / 1e9:.0f} GB available)"}
+        rotating = True
+    else:
+        rotating = False
+    t_plan = time.perf_counter()
+    if nchunks == 1:
+        cobs, cplans = [obs], [plan]
+    else:
+        cobs = [obs.select(np.arange(nbl), chunk_T, k * chunk_T) for k in range(nchunks)]
+        cplans = [idg.Plan.from_observation(o) for o in cobs]
+    plan_s = time.perf_counter() - t_plan
+    # A-term slots of every chunk (slot boundaries are cut to the chunk window)
+    first_slot = [int(np.searchsorted(obs.aterm_offsets, k * chunk_T, side="right")) - 1 for k in range(nchunks)]
+    # union of the covered grid rows of all chunk plans (the band the collectives move)
+    rows = None
+    if world > 1:
+        ys = np.concatenate([p.metadata()["y"] for p in cplans])
+        rows = parallel.union_rows(parallel.coverage_rows(ys, obs.subgrid_size, obs.grid_size), device=dev)
+
+    # host buffers: [chunk][nbl][chunk_T][C][4] (chunk-major), or 2 rotating chunk buffers per direction
+    nbuf = 2 if rotating else nchunks
+    regs = []
+    def alloc(n):
+        t, reg = host_buffer((n, nbl, chunk_T, C, 4), torch.complex64)
+        if reg:
+            regs.append(t)
+        return t
+    in_h = alloc(nbuf) if n_in else None
+    out_h = alloc(nbuf)
+    uvw_h, reg = host_buffer((nchunks, nbl, chunk_T, 3), torch.float32)
+    if reg:
+        regs.append(uvw_h)
+    for k in range(nchunks):
+        uvw_h[k].copy_(torch.from_numpy(cobs[k].uvw))
+    at_h = torch.from_numpy(aterms).pin_memory()
+    model_h = grid_d.cpu().pin_memory() if kind == "degrid" else None
+    chk_ref = None
+    if kind == "grid+degrid":
+        for k in range(nbuf):
+            in_h[k].copy_(vis_d[:, k * chunk_T:(k + 1) * chunk_T])
+    elif nchunks == 1:
+        chk_ref = None   # compared after the loop against the device path's predictions (same plan)
+    if kind == "degrid" and nchunks == 1:
+        nb_chk = min(64, nbl)
+        chk_ref = out_d[:nb_chk].cpu()
+    del vis_d, out_d
+    torch.cuda.empty_cache()
+    # one workspace, grid, uvw and A-term buffer per stream: a workspace serves one in-flight call
+    wss = [idg.workspace(cplans[0], dev, full=True) for _ in range(2)]
+    streams = [stream, torch.cuda.Stream(dev)]
+    grids = [grid_d, torch.zeros_like(grid_d)]
+    uvws = [torch.empty((nchunks, nbl, chunk_T, 3), dtype=torch.float32, device=dev) for _ in range(2)]
+    ats = [torch.empty_like(torch.from_numpy(aterms), device=dev) for _ in range(2)]
+    tp_d = torch.from_numpy(taper).to(dev)
+
+    def e2e_step(k):
+        j = k % 2
+        s_k, g_k, u_k, a_k, w_k, o_k = streams[j], grids[j], uvws[j], ats[j], wss[j], out_h
+        with torch.cuda.stream(s_k):
+            u_k.copy_(uvw_h, non_blocking=True)
+            a_k.copy_(at_h, non_blocking=True)
+            if kind == "grid+degrid":
+                g_k.zero_()
+                for c in range(nchunks):
+                    sl = slice(first_slot[c], first_slot[c] + cobs[c].nr_aterm_slots)
+                    idg.grid_host(cplans[c], in_h[c % nbuf], u_k[c], a_k[sl], tp_d, g_k, w_k, stream=s_k)
+                parallel.reduce_grid(g_k, dst=0, rows=rows)
+            elif rank == 0:
+                g_k.copy_(model_h, non_blocking=True)
+            parallel.broadcast_grid(g_k, src=0, rows=rows)
+            for c in range(nchunks):
+                sl = slice(first_slot[c], first_slot[c] + cobs[c].nr_aterm_slots)
+                idg.degrid_host(cplans[c], g_k, u_k[c], a_k[sl], tp_d, o_k[c % nbuf], w_k, stream=s_k)
+
+    e2e_step(0)
+    e2e_step(1)
+    barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ksteps = max(1, min(args.steps, args.e2e_steps))
+    e0.record(stream)
+    streams[1].wait_event(e0)
+    for k in range(ksteps):
+        e2e_step(k)
+    last = torch.cuda.Event()
+    last.record(streams[1])
+    stream.wait_event(last)
+    e1.record(stream)
+    barrier()
+    te = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    check = None
+    out_last = out_h
+    if kind == "grid+degrid" and not rotating and world == 1:
+        # whole-data check: degrid = grid^H, so <vis, degrid(grid(vis))> = ||grid(vis)||^2 (adjoint identity)
+        lhs = vdot_chunked(in_h, out_last, dev)
+        g = grids[(ksteps - 1) % 2]
+        rhs = float(torch.linalg.vector_norm(g.view(torch.float32).to(torch.float64)) ** 2)
+        check = {"adjoint_identity_rel_err": abs(lhs - rhs) / abs(rhs)}
+    elif chk_ref is not None:
+        got = out_last[0, :chk_ref.shape[0]]
+        check = {"rel_rms_vs_device_path": float(torch.linalg.vector_norm(got - chk_ref) /
+                                                 torch.linalg.vector_norm(chk_ref))}
+    h2d = (n_in * nbl * T * C * 32 + uvw_h.numel() * 4 + at_h.numel() * 8 +
+           (model_h.numel() * 8 if model_h is not None and rank == 0 else 0))
+    res = {"value": nvis_total * ksteps / (float(te.item()) * 1e-3) / 1e6, "unit": "MVis/s",
+           "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(nbl * T * C * 32), "steps": ksteps,
+           "time_chunks": nchunks, "chunk_timesteps": chunk_T, "chunk_plans_s": plan_s,
+           "host_buffers": ("2 rotating chunk buffers per direction (host memory); every chunk still crosses "
+                            "PCIe each step") if rotating else "full page-locked host arrays",
+           "check": check,
+           "api": "idg_grid_host + idg_degrid_host (host-streamed work groups, one staging buffer per work "
+                  "group; independent steps on two alternating streams so the uploads of step k+1 overlap the "
+                  "degridding and downloads of step k)"}
+    for t in regs:
+        unregister_host(t)
+    return res
+
+
 def main():
     ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="lofar", choices=sorted(CONFIG_NAMES))
+    ap.add_argument("--config", default="ska", choices=sorted(CONFIG_NAMES),
+                    help="default: the SKA-low-shaped set on an 8192^2 grid (configs[3], the north star's target)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=8)
+    ap.add_argument("--e2e-steps", type=int, default=6)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-baseline-s", type=float, default=15.0)
     ap.add_argument("--reference-step-s", type=float, default=8.0)
     ap.add_argument("--rho-iterations", type=int, default=16384)
-    ap.add_argument("--rho-sweep", action="store_true")
+    ap.add_argument("--no-rho-sweep", action="store_true")
+    ap.add_argument("--no-kernel-energy", action="store_true")
+    ap.add_argument("--energy-launches", type=int, default=5)
     ap.add_argument("--timesteps", type=int, default=0,
                     help="tuning only: override the config's T (the line then names the reduced workload)")
     args = ap.parse_args()

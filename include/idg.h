@@ -169,11 +169,16 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
  * current device: every sincos evaluation is followed by rho-1 FMAs plus the one FMA that forms its
  * argument (rho FMAs per sincos).  ops = 2 per FMA + 1 per sin + 1 per cos (op definition).
  *   rho in {0,1,2,3,4,6,8,12,16,17,20,24,32,48,64}; rho = 0 measures sincos alone (2 ops each: the
- *   XU/MUFU bound of the tensor-core kernels, whose multiply-adds run on the tensor cores);  iterations >= 1 (work per thread);  ops_per_second receives the measured
+ *   XU/MUFU bound);  iterations >= 1 (work per thread);  ops_per_second receives the measured
  *   throughput (synchronous: the call waits for the kernel; timed with CUDA events on `stream`).
+ * The FMAs of two units run as one packed f32x2 FFMA2 (the B200 FMA-pipe form);
+ * idg_rho_benchmark_scalar issues them as scalar 3-register FFMA (the paper's form, which sm_100 issues
+ * at half the FP32 lane rate).
  */
 idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream,
                              double *ops_per_second, double *seconds);
+idg_status idg_rho_benchmark_scalar(int32_t rho, int32_t iterations, idg_stream stream,
+                                    double *ops_per_second, double *seconds);
 
 /*
  * Kernel timing (measurement only).  When enabled, every kernel the library launches is bracketed

@@ -688,8 +688,8 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
 }
 #undef IDG_PIPE
 
-idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
-                             double *seconds) {
+static idg_status rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
+                                double *seconds, bool packed) {
     static const int kSupported[] = {0, 1, 2, 3, 4, 6, 8, 12, 16, 17, 20, 24, 32, 48, 64};
     if (std::find(std::begin(kSupported), std::end(kSupported), rho) == std::end(kSupported) ||
         iterations < 1 || !ops_per_second)
@@ -699,22 +699,20 @@ idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream,
     float *d_out = nullptr;
     cudaError_t e = cudaMalloc(&d_out, sizeof(float) * 148 * 64 * 256);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(rho)");
-    cudaEvent_t e0, e1;
-    cudaEventCreate(&e0);
-    cudaEventCreate(&e1);
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
     int blocks = 0, threads = 0, units = 0;
-    // warm-up launch, then the timed one
-    e = idg::launch_rho_benchmark(rho, std::max(1, iterations / 8), d_out, s, &blocks, &threads, &units);
-    if (e == cudaSuccess) {
-        cudaEventRecord(e0, s);
-        e = idg::launch_rho_benchmark(rho, iterations, d_out, s, &blocks, &threads, &units);
-        cudaEventRecord(e1, s);
+    if ((e = cudaEventCreate(&e0)) == cudaSuccess && (e = cudaEventCreate(&e1)) == cudaSuccess) {
+        // warm-up launch, then the timed one
+        e = idg::launch_rho_benchmark(rho, std::max(1, iterations / 8), d_out, s, &blocks, &threads, &units, packed);
+        if (e == cudaSuccess) e = cudaEventRecord(e0, s);
+        if (e == cudaSuccess) e = idg::launch_rho_benchmark(rho, iterations, d_out, s, &blocks, &threads, &units, packed);
+        if (e == cudaSuccess) e = cudaEventRecord(e1, s);
     }
     if (e == cudaSuccess) e = cudaEventSynchronize(e1);
     float ms = 0.0f;
     if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, e0, e1);
-    cudaEventDestroy(e0);
-    cudaEventDestroy(e1);
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
     cudaFree(d_out);
     if (e != cudaSuccess) return cuda_fail(e, "rho benchmark");
     const double sincos = double(blocks) * threads * units * double(iterations);
@@ -722,6 +720,16 @@ idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream,
     *ops_per_second = ops / (double(ms) * 1e-3);
     if (seconds) *seconds = double(ms) * 1e-3;
     return IDG_OK;
+}
+
+idg_status idg_rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
+                             double *seconds) {
+    return rho_benchmark(rho, iterations, stream, ops_per_second, seconds, true);
+}
+
+idg_status idg_rho_benchmark_scalar(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
+                                    double *seconds) {
+    return rho_benchmark(rho, iterations, stream, ops_per_second, seconds, false);
 }
 
 idg_status idg_profiling_enable(int32_t enable) {

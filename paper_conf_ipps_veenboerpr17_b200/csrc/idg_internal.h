@@ -77,7 +77,7 @@ const char *variant_names(int which);
 cudaError_t launch_zero_ranges(float2 *vis, const int64_t *ranges, int64_t nr, int64_t base, cudaStream_t s);
 const char *last_variant(int which);   // name of the variant the last launch used ("" before any)
 cudaError_t launch_rho_benchmark(int rho, int iterations, float *d_out, cudaStream_t s,
-                                 int *blocks, int *threads, int *units_per_thread);
+                                 int *blocks, int *threads, int *units_per_thread, bool packed);
 
 // Kernel-launch bookkeeping (profiling + launch counter), idg_api.cpp.
 struct LaunchScope {

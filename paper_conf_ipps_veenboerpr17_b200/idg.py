@@ -45,6 +45,7 @@ _lib = None
 
 EXPORTED = ["idg_plan_create", "idg_plan_destroy", "idg_plan_nr_subgrids", "idg_plan_metadata",
             "idg_plan_stats", "idg_workspace_size", "idg_grid", "idg_degrid", "idg_rho_benchmark",
+            "idg_rho_benchmark_scalar",
             "idg_profiling_enable", "idg_profiling_reset", "idg_profiling_read", "idg_launch_count",
             "idg_kernel_variants", "idg_host_workspace_size", "idg_grid_host", "idg_degrid_host",
             "idg_status_string", "idg_last_error", "idg_last_variant"]
@@ -72,8 +73,8 @@ def lib() -> ctypes.CDLL:
     L.idg_host_workspace_size.argtypes = [P, ctypes.POINTER(sz)]
     L.idg_grid_host.argtypes = [P, P, P, P, P, P, P, sz, P]
     L.idg_degrid_host.argtypes = [P, P, P, P, P, P, P, sz, P]
-    L.idg_rho_benchmark.argtypes = [i32, i32, P, ctypes.POINTER(ctypes.c_double),
-                                    ctypes.POINTER(ctypes.c_double)]
+    for f in ("idg_rho_benchmark", "idg_rho_benchmark_scalar"):
+        getattr(L, f).argtypes = [i32, i32, P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
     L.idg_profiling_enable.argtypes = [i32]
     L.idg_profiling_read.argtypes = [ctypes.POINTER(KernelTime), i32, ctypes.POINTER(i32)]
     L.idg_launch_count.restype = i64
@@ -298,11 +299,12 @@ def degrid_host(plan: Plan, grid_in, uvw, aterms, taper, vis_host_out, ws, strea
     return vis_host_out
 
 
-def rho_benchmark(rho: int = 17, iterations: int = 4096, stream=None) -> tuple[float, float]:
-    """The paper's FMA:sincos benchmark: returns (ops/s, seconds) at ratio rho."""
+def rho_benchmark(rho: int = 17, iterations: int = 4096, stream=None, scalar: bool = False) -> tuple[float, float]:
+    """The paper's FMA:sincos benchmark: returns (ops/s, seconds) at ratio rho.  FMAs as packed
+    FFMA2 pairs (B200 form), or as scalar FFMA with scalar=True (the paper's form)."""
     ops, sec = ctypes.c_double(), ctypes.c_double()
-    _check(lib().idg_rho_benchmark(int(rho), int(iterations), _stream(stream), ctypes.byref(ops),
-                                   ctypes.byref(sec)), "idg_rho_benchmark")
+    f = lib().idg_rho_benchmark_scalar if scalar else lib().idg_rho_benchmark
+    _check(f(int(rho), int(iterations), _stream(stream), ctypes.byref(ops), ctypes.byref(sec)), "idg_rho_benchmark")
     return ops.value, sec.value
 
 

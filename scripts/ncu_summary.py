@@ -9,6 +9,7 @@ import csv
 import io
 import json
 import os
+import re
 import subprocess
 from collections import defaultdict
 
@@ -60,6 +61,28 @@ def summarize(rep):
                 u, v = d[k]
                 b += float(v.replace(",", "")) * SCALE.get(u, 1)
         rec["dram_bytes"] = b
+        # per-pipe utilisation: instructions issued to a pipe and cycles the pipe was busy, both as % of its
+        # peak (ComputeWorkloadAnalysis); the binding pipe is the busiest of them
+        pipes = {}
+        for h, (u, v) in d.items():
+            m = re.match(r"^sm__(inst_executed_pipe|pipe)_([a-z0-9_]+?)(_cycles_active)?"
+                         r"\.avg\.pct_of_peak_sustained_active$", h)
+            if not m:
+                continue
+            try:
+                val = float(v.replace(",", ""))
+            except ValueError:
+                continue
+            key = ("inst:" if m.group(1) == "inst_executed_pipe" else "cycles:") + m.group(2)
+            pipes[key] = val
+        if pipes:
+            rec["pipes %"] = ", ".join(f"{k} {v:.1f}" for k, v in sorted(pipes.items(), key=lambda x: -x[1])[:12])
+            bk = max(pipes, key=pipes.get)
+            rec["binding pipe"] = f"{bk} {pipes[bk]:.1f}%"
+            rec["_pipes"] = pipes
+        ia = d.get("smsp__issue_active.avg.pct_of_peak_sustained_active")
+        if ia:
+            rec["_issue"] = float(ia[1].replace(",", ""))
         res.append(rec)
     return res
 
@@ -100,13 +123,19 @@ def main():
         for rec in summarize(rep):
             md.append(f"## {rec['kernel']}  ({os.path.basename(rep)})")
             for k, v in rec.items():
-                if k != "kernel":
+                if k != "kernel" and not k.startswith("_"):
                     md.append(f"- {k}: {v}")
             md.append("")
             short = "degridder" if "degridder" in rec["kernel"] else "gridder" if "gridder" in rec["kernel"] \
                 else rec["kernel"].split("(")[0]
-            js.setdefault(args.config, {})[short] = {"tag": args.tag, "kernel": rec["kernel"],
-                                                     "dram_bytes": rec["dram_bytes"]}
+            ent = {"tag": args.tag, "kernel": rec["kernel"], "dram_bytes": rec["dram_bytes"]}
+            if "_pipes" in rec:
+                p = rec["_pipes"]
+                bk = max(p, key=p.get)
+                ent.update({"binding_pipe": bk, "binding_pipe_frac": p[bk] / 100.0,
+                            "issue_active_frac": rec.get("_issue", 0.0) / 100.0,
+                            "pipes_pct_of_peak": dict(sorted(p.items(), key=lambda x: -x[1]))})
+            js.setdefault(args.config, {})[short] = ent
     if args.launches:
         md += ["## launch list (ncu gpu__time_duration, cold/serialised: compare shares)", "",
                "| kernel | launches | total ms | share |", "|---|---|---|---|"]

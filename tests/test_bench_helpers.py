@@ -24,3 +24,14 @@ def test_sincos_per_pair_by_family():
 def test_ops_per_pair_is_the_papers():
     # 17 FMA + 1 sincos = 36 paper-ops per (pixel, visibility) pair
     assert bench.OPS_PER_PAIR == 36
+
+
+def test_sincos_fma_roofline_unit_counts():
+    # 148 SMs x min(128/17, 16/2) pairs/clk x 36 ops at 1965 MHz = 78.8 TOps/s
+    assert abs(bench.sincos_fma_roofline(1965) - 78.84) < 0.05
+
+
+def test_step_kind_per_config():
+    assert bench.STEP_KIND["predict"] == "degrid"                  # configs[4]: degridding-only sweep
+    assert all(bench.STEP_KIND[c] == "grid+degrid" for c in ("tiny", "lofar", "lofar_dde", "ska"))
+    assert bench.E2E_TIME_CHUNK["ska"] == 1024                      # 8 chunks of 1024
