@@ -593,16 +593,19 @@ def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, wo
         chk_ref = out_d[:nb_chk].cpu()
     del vis_d, out_d
     torch.cuda.empty_cache()
-    # one workspace, grid, uvw and A-term buffer per stream: a workspace serves one in-flight call
-    wss = [idg.workspace(cplans[0], dev, full=True) for _ in range(2)]
-    streams = [stream, torch.cuda.Stream(dev)]
-    grids = [grid_d, torch.zeros_like(grid_d)]
-    uvws = [torch.empty((nchunks, nbl, chunk_T, 3), dtype=torch.float32, device=dev) for _ in range(2)]
-    ats = [torch.empty_like(torch.from_numpy(aterms), device=dev) for _ in range(2)]
+    # one workspace, grid, uvw and A-term buffer per stream: a workspace serves one in-flight call.  Steps
+    # rotate over NS streams: a host-streamed call starts its uploads after the work queued before it on its
+    # stream (the caller's ordering), so with NS streams step k+1's uploads wait only for step k+1-NS.
+    NS = 3
+    wss = [idg.workspace(cplans[0], dev, max_buffers=32) for _ in range(NS)]
+    streams = [stream] + [torch.cuda.Stream(dev) for _ in range(NS - 1)]
+    grids = [grid_d] + [torch.zeros_like(grid_d) for _ in range(NS - 1)]
+    uvws = [torch.empty((nchunks, nbl, chunk_T, 3), dtype=torch.float32, device=dev) for _ in range(NS)]
+    ats = [torch.empty_like(torch.from_numpy(aterms), device=dev) for _ in range(NS)]
     tp_d = torch.from_numpy(taper).to(dev)
 
     def e2e_step(k):
-        j = k % 2
+        j = k % NS
         s_k, g_k, u_k, a_k, w_k, o_k = streams[j], grids[j], uvws[j], ats[j], wss[j], out_h
         with torch.cuda.stream(s_k):
             u_k.copy_(uvw_h, non_blocking=True)
@@ -620,18 +623,20 @@ def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, wo
                 sl = slice(first_slot[c], first_slot[c] + cobs[c].nr_aterm_slots)
                 idg.degrid_host(cplans[c], g_k, u_k[c], a_k[sl], tp_d, o_k[c % nbuf], w_k, stream=s_k)
 
-    e2e_step(0)
-    e2e_step(1)
+    for k in range(NS):
+        e2e_step(k)
     barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ksteps = max(1, min(args.steps, args.e2e_steps))
     e0.record(stream)
-    streams[1].wait_event(e0)
+    for s_ in streams[1:]:
+        s_.wait_event(e0)
     for k in range(ksteps):
         e2e_step(k)
-    last = torch.cuda.Event()
-    last.record(streams[1])
-    stream.wait_event(last)
+    for s_ in streams[1:]:
+        last = torch.cuda.Event()
+        last.record(s_)
+        stream.wait_event(last)
     e1.record(stream)
     barrier()
     te = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
@@ -642,7 +647,7 @@ def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, wo
     if kind == "grid+degrid" and not rotating and world == 1:
         # whole-data check: degrid = grid^H, so <vis, degrid(grid(vis))> = ||grid(vis)||^2 (adjoint identity)
         lhs = vdot_chunked(in_h, out_last, dev)
-        g = grids[(ksteps - 1) % 2]
+        g = grids[(ksteps - 1) % NS]
         rhs = float(torch.linalg.vector_norm(g.view(torch.float32).to(torch.float64)) ** 2)
         check = {"adjoint_identity_rel_err": abs(lhs - rhs) / abs(rhs)}
     elif chk_ref is not None:
@@ -657,8 +662,8 @@ def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, wo
            "host_buffers": ("2 rotating chunk buffers per direction (host memory); every chunk still crosses "
                             "PCIe each step") if rotating else "full page-locked host arrays",
            "check": check,
-           "api": "idg_grid_host + idg_degrid_host (host-streamed work groups, one staging buffer per work "
-                  "group; independent steps on two alternating streams so the uploads of step k+1 overlap the "
+           "api": "idg_grid_host + idg_degrid_host (host-streamed work groups through <= 32 staging buffers "
+                  "per direction; independent steps rotate over 3 streams so the uploads of step k+1 overlap the "
                   "degridding and downloads of step k)"}
     for t in regs:
         unregister_host(t)

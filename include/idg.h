@@ -165,6 +165,32 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
                            size_t workspace_bytes, idg_stream stream);
 
 /*
+ * Host adder / splitter: the grid lives in HOST memory (Section V-C-e, option 2: "copy the subgrids
+ * into host memory and perform the operation on the CPU ... only required when dealing with large images
+ * that no longer fit into GPU device memory").  Visibilities are in host memory as for idg_grid_host.
+ * Per work group the kernels write (gridding) or read (degridding) the group's transformed subgrids in a
+ * device buffer instead of the grid; the subgrids stream to / from page-locked host buffers (allocated by
+ * the library per workspace, freed with the plan) and host threads (IDG_HOST_THREADS, default: the
+ * hardware concurrency, at most 32) add them into / split them out of the host grid -- each thread owns
+ * the grid rows r with r mod T == its index, so no atomics -- while the GPU processes the next groups.
+ *   idg_grid_host_adder      h_vis (read) -> h_grid complex64 [nz][4][N][N] HOST, ACCUMULATED (+=).
+ *                            Returns when h_grid holds the result (the host adds are done); later work
+ *                            on `stream` may reuse the workspace.
+ *   idg_degrid_host_splitter h_grid (read) -> h_vis OVERWRITTEN (dropped visibilities = 0).  Waits for
+ *                            the caller's earlier work on `stream` before reading h_grid; asynchronous
+ *                            afterwards: h_vis is complete when `stream` reaches the call's end.
+ * d_workspace must hold idg_host_adder_workspace_size() bytes (3 staging buffers per direction, each
+ * one work group's visibilities + subgrids); a larger workspace gives more buffers.  Errors as idg_grid.
+ */
+idg_status idg_host_adder_workspace_size(const idg_plan *plan, size_t *bytes);
+idg_status idg_grid_host_adder(const idg_plan *plan, const void *h_vis, const float *d_uvw,
+                               const void *d_aterms, const float *d_taper, void *h_grid, void *d_workspace,
+                               size_t workspace_bytes, idg_stream stream);
+idg_status idg_degrid_host_splitter(const idg_plan *plan, const void *h_grid, const float *d_uvw,
+                                    const void *d_aterms, const float *d_taper, void *h_vis,
+                                    void *d_workspace, size_t workspace_bytes, idg_stream stream);
+
+/*
  * idg_rho_benchmark -- the paper's FMA:sincos throughput benchmark (Fig. 12) on the
  * current device: every sincos evaluation is followed by rho-1 FMAs plus the one FMA that forms its
  * argument (rho FMAs per sincos).  ops = 2 per FMA + 1 per sin + 1 per cos (op definition).

@@ -4,6 +4,10 @@
 #include <algorithm>
 #include <atomic>
 #include <cmath>
+#include <complex>
+#include <condition_variable>
+#include <functional>
+#include <thread>
 #include <cstdio>
 #include <cstring>
 #include <cstdlib>
@@ -44,16 +48,83 @@ std::map<std::string, std::pair<int64_t, double>> g_prof_totals;
 constexpr int kStagingBuffers = 3;                  // triple buffering (Fig. 7)
 constexpr size_t kHostChunkBytes = size_t(128) << 20;  // visibilities per work group (host-streamed calls)
 
-// Events of the host-streamed pipeline for one workspace (its staging buffers), grown on demand.
+// Events of the host-streamed pipeline for one workspace (its staging buffers), grown on demand, and the
+// page-locked host subgrid buffers of the host adder / splitter.
 struct PipeEvents {
     cudaEvent_t entry = nullptr;                              // the caller's stream at call entry
     std::vector<cudaEvent_t> h2d, kernel_g, kernel_d, d2h;    // per staging buffer
+    std::vector<void *> host_subgrids;                        // [buffer] pinned, host_subgrid_bytes each
+    size_t host_subgrid_bytes = 0;
     ~PipeEvents() {
         if (entry) cudaEventDestroy(entry);
         for (auto *v : {&h2d, &kernel_g, &kernel_d, &d2h})
             for (cudaEvent_t ev : *v) cudaEventDestroy(ev);
+        for (void *p : host_subgrids) cudaFreeHost(p);
     }
 };
+
+// A fixed pool of host threads for the host adder / splitter: run(f) calls f(thread, nthreads) on every
+// thread and returns when all are done.
+class HostPool {
+  public:
+    explicit HostPool(int n) : n_(std::max(1, n)) {
+        for (int t = 1; t < n_; ++t) threads_.emplace_back([this, t] { loop(t); });
+    }
+    ~HostPool() {
+        {
+            std::lock_guard<std::mutex> l(mu_);
+            stop_ = true;
+            ++gen_;
+        }
+        cv_.notify_all();
+        for (auto &th : threads_) th.join();
+    }
+    void run(const std::function<void(int, int)> &f) {
+        {
+            std::lock_guard<std::mutex> l(mu_);
+            job_ = &f;
+            pending_ = n_ - 1;
+            ++gen_;
+        }
+        cv_.notify_all();
+        f(0, n_);
+        std::unique_lock<std::mutex> l(mu_);
+        done_cv_.wait(l, [this] { return pending_ == 0; });
+        job_ = nullptr;
+    }
+    int size() const { return n_; }
+
+  private:
+    void loop(int t) {
+        uint64_t seen = 0;
+        for (;;) {
+            const std::function<void(int, int)> *job;
+            {
+                std::unique_lock<std::mutex> l(mu_);
+                cv_.wait(l, [&] { return gen_ != seen; });
+                seen = gen_;
+                if (stop_) return;
+                job = job_;
+            }
+            (*job)(t, n_);
+            std::lock_guard<std::mutex> l(mu_);
+            if (--pending_ == 0) done_cv_.notify_one();
+        }
+    }
+    int n_;
+    std::vector<std::thread> threads_;
+    std::mutex mu_;
+    std::condition_variable cv_, done_cv_;
+    const std::function<void(int, int)> *job_ = nullptr;
+    int pending_ = 0;
+    uint64_t gen_ = 0;
+    bool stop_ = false;
+};
+
+int host_threads() {
+    if (const char *env = std::getenv("IDG_HOST_THREADS")) return std::max(1, std::atoi(env));
+    return int(std::max(1u, std::min(32u, std::thread::hardware_concurrency())));
+}
 
 struct DeviceCopy {
     idg_metadata *items = nullptr;
@@ -96,6 +167,7 @@ struct idg_plan {
                                      // split at baseline boundaries (R-12, R-13: predicted as 0)
     std::vector<WorkGroup> groups;   // host-streamed work groups
     size_t group_bytes = 0;          // largest work group's visibility bytes
+    int64_t group_items = 0;         // most work items in a work group (host adder / splitter)
     int32_t channel_gcd = 1;
     int32_t channels_uniform = 0;
     float channel_step = 0.0f;
@@ -441,6 +513,7 @@ idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, i
                 while (r < nr && plan->dropped[2 * r] < int64_t(b1) * vis_per_bl) ++r;
                 plan->groups.push_back(WorkGroup{b0, b1, i0, it, r0, r});
                 plan->group_bytes = std::max(plan->group_bytes, size_t(b1 - b0) * bl_bytes);
+                plan->group_items = std::max(plan->group_items, it - i0);
             }
         }
         plan->order.resize(plan->items.size());
@@ -687,6 +760,232 @@ idg_status idg_degrid_host(const idg_plan *plan, const void *d_grid, const float
     }
 }
 #undef IDG_PIPE
+
+}  // extern "C"
+
+// ------------------------------------------------------------------------------------------------
+// Host adder / splitter (Section V-C-e, option 2): "copy the subgrids into host memory and perform
+// the operation on the CPU ... required when dealing with large images that no longer fit into GPU device
+// memory".  The grid lives in HOST memory; the kernels write (gridding) or read (degridding) the work
+// group's transformed subgrids in a device buffer, which streams to / from page-locked host buffers; host
+// threads add them into (or split them out of) the host grid while the GPU works on the next groups.
+// ------------------------------------------------------------------------------------------------
+namespace {
+
+size_t subgrid_bytes(const idg_plan *plan) { return size_t(4) * plan->params.subgrid_size * plan->params.subgrid_size * 8; }
+size_t adder_buffer_bytes(const idg_plan *plan) {   // one staging buffer: visibilities + subgrids of a work group
+    return plan->group_bytes + size_t(plan->group_items) * subgrid_bytes(plan);
+}
+
+// page-locked host subgrid buffers (n of them) of a workspace's pipeline
+cudaError_t host_subgrid_buffers(PipeEvents *pe, int n, size_t bytes) {
+    if (pe->host_subgrid_bytes < bytes) {
+        for (void *p : pe->host_subgrids) cudaFreeHost(p);
+        pe->host_subgrids.clear();
+        pe->host_subgrid_bytes = bytes;
+    }
+    while (int(pe->host_subgrids.size()) < n) {
+        void *p = nullptr;
+        cudaError_t e = cudaHostAlloc(&p, std::max<size_t>(1, bytes), cudaHostAllocDefault);
+        if (e != cudaSuccess) return e;
+        pe->host_subgrids.push_back(p);
+    }
+    return cudaSuccess;
+}
+
+// grid[z][pol][y + ky][x + kx] (+)= sub[j][pol][ky][kx] for the items [i0, i1); rows interleaved over threads
+// (row r -> thread r mod T), so no two threads touch the same grid row and no atomics are needed.
+void host_add_or_split(const idg_plan *plan, HostPool &pool, int64_t i0, int64_t i1, std::complex<float> *grid,
+                       std::complex<float> *sub, bool add) {
+    const int ns = plan->params.subgrid_size;
+    const int64_t N = plan->params.grid_size;
+    pool.run([&](int t, int T) {
+        for (int64_t j = i0; j < i1; ++j) {
+            const idg_metadata &m = plan->items[size_t(j)];
+            std::complex<float> *s = sub + (j - i0) * 4 * ns * ns;
+            int ky0 = int(((int64_t(t) - m.y) % T + T) % T);
+            for (int ky = ky0; ky < ns; ky += T)
+                for (int pol = 0; pol < 4; ++pol) {
+                    std::complex<float> *g = grid + ((int64_t(m.z) * 4 + pol) * N + m.y + ky) * N + m.x;
+                    std::complex<float> *r = s + (int64_t(pol) * ns + ky) * ns;
+                    if (add)
+                        for (int kx = 0; kx < ns; ++kx) g[kx] += r[kx];
+                    else
+                        std::memcpy(r, g, size_t(ns) * sizeof(std::complex<float>));
+                }
+        }
+    });
+}
+
+}  // namespace
+
+extern "C" {
+
+idg_status idg_host_adder_workspace_size(const idg_plan *plan, size_t *bytes) {
+    if (!plan || !bytes) return fail(IDG_ERR_INVALID_ARG, "NULL argument");
+    *bytes = size_t(2) * kStagingBuffers * adder_buffer_bytes(plan);
+    return IDG_OK;
+}
+
+#define IDG_PIPE(call)                      \
+    do {                                    \
+        if ((e = (call)) != cudaSuccess) {  \
+            what = #call;                   \
+            goto pipe_error;                \
+        }                                   \
+    } while (0)
+
+idg_status idg_grid_host_adder(const idg_plan *plan, const void *h_vis, const float *d_uvw, const void *d_aterms,
+                               const float *d_taper, void *h_grid, void *d_workspace, size_t workspace_bytes,
+                               idg_stream stream) {
+    try {
+        idg_status st = validate_call(plan, h_vis, d_uvw, d_aterms, d_taper, h_grid);
+        if (st != IDG_OK || plan->items.empty()) return st;
+        const size_t per = adder_buffer_bytes(plan);
+        if (!d_workspace || workspace_bytes < size_t(2) * kStagingBuffers * per)
+            return fail(IDG_ERR_WORKSPACE_TOO_SMALL, "idg_grid_host_adder needs idg_host_adder_workspace_size() = " +
+                                                         std::to_string(size_t(2) * kStagingBuffers * per) + " bytes");
+        const DeviceCopy *dc = nullptr;
+        if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        std::lock_guard<std::mutex> lock(*dc->pipeline_mu);
+        const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+        const size_t bl_bytes = size_t(plan->nr_timesteps) * plan->nr_channels * 32;
+        const int64_t bl_f2 = int64_t(plan->nr_timesteps) * plan->nr_channels * 4;
+        const size_t sgb = subgrid_bytes(plan);
+        const int nb = int(std::max<size_t>(kStagingBuffers, std::min(workspace_bytes / (2 * per), plan->groups.size())));
+        char *base = static_cast<char *>(d_workspace);        // grid half: [nb][vis | subgrids]
+        const char *what = "";
+        PipeEvents *pe = nullptr;
+        cudaError_t e = pipe_events(dc, d_workspace, nb, &pe);
+        if (e == cudaSuccess) e = host_subgrid_buffers(pe, 2 * nb, size_t(plan->group_items) * sgb);
+        if (e != cudaSuccess) return cuda_fail(e, "idg_grid_host_adder: events / host buffers");
+        HostPool pool(host_threads());
+        auto *grid = static_cast<std::complex<float> *>(h_grid);
+        auto drain = [&](size_t gj) -> cudaError_t {   // host-add work group gj once its subgrids have arrived
+            const int b = int(gj % nb);
+            cudaError_t err = cudaEventSynchronize(pe->d2h[b]);
+            if (err != cudaSuccess) return err;
+            host_add_or_split(plan, pool, plan->groups[gj].i0, plan->groups[gj].i1, grid,
+                              static_cast<std::complex<float> *>(pe->host_subgrids[b]), true);
+            return cudaSuccess;
+        };
+        IDG_PIPE(cudaEventRecord(pe->entry, s));
+        IDG_PIPE(cudaStreamWaitEvent(dc->h2d, pe->entry, 0));
+        for (size_t gi = 0; gi < plan->groups.size(); ++gi) {
+            const WorkGroup &g = plan->groups[gi];
+            const int b = int(gi % nb);
+            char *vbuf = base + size_t(b) * per;
+            auto *sbuf = reinterpret_cast<float2 *>(vbuf + plan->group_bytes);
+            if (gi >= size_t(nb)) IDG_PIPE(drain(gi - nb));   // frees host buffer b (and overlaps the GPU)
+            IDG_PIPE(cudaStreamWaitEvent(dc->h2d, pe->kernel_g[b], 0));
+            IDG_PIPE(cudaMemcpyAsync(vbuf, static_cast<const char *>(h_vis) + size_t(g.b0) * bl_bytes,
+                                     size_t(g.b1 - g.b0) * bl_bytes, cudaMemcpyHostToDevice, dc->h2d));
+            IDG_PIPE(cudaEventRecord(pe->h2d[b], dc->h2d));
+            IDG_PIPE(cudaStreamWaitEvent(s, pe->h2d[b], 0));
+            IDG_PIPE(cudaStreamWaitEvent(s, pe->d2h[b], 0));  // the subgrid buffer's previous download
+            if (g.i1 > g.i0) {
+                idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper,
+                                              reinterpret_cast<float2 *>(vbuf) - int64_t(g.b0) * bl_f2, nullptr);
+                a.subgrids = sbuf;
+                a.order = dc->iota + g.i0;
+                a.nr_items = g.i1 - g.i0;
+                IDG_PIPE(idg::launch_gridder(a, s));
+            }
+            IDG_PIPE(cudaEventRecord(pe->kernel_g[b], s));
+            IDG_PIPE(cudaStreamWaitEvent(dc->d2h, pe->kernel_g[b], 0));
+            if (g.i1 > g.i0)
+                IDG_PIPE(cudaMemcpyAsync(pe->host_subgrids[b], sbuf, size_t(g.i1 - g.i0) * sgb,
+                                         cudaMemcpyDeviceToHost, dc->d2h));
+            IDG_PIPE(cudaEventRecord(pe->d2h[b], dc->d2h));
+        }
+        for (size_t gi = plan->groups.size() > size_t(nb) ? plan->groups.size() - nb : 0; gi < plan->groups.size(); ++gi)
+            IDG_PIPE(drain(gi));
+        return IDG_OK;
+    pipe_error:
+        return cuda_fail(e, std::string("idg_grid_host_adder: ") + what);
+    } catch (const std::exception &ex) {
+        return fail(IDG_ERR_INVALID_ARG, ex.what());
+    }
+}
+
+idg_status idg_degrid_host_splitter(const idg_plan *plan, const void *h_grid, const float *d_uvw,
+                                    const void *d_aterms, const float *d_taper, void *h_vis, void *d_workspace,
+                                    size_t workspace_bytes, idg_stream stream) {
+    try {
+        idg_status st = validate_call(plan, h_vis, d_uvw, d_aterms, d_taper, h_grid);
+        if (st != IDG_OK) return st;
+        if (plan->items.empty())   // everything dropped: the host-streamed degridder defines it as 0
+            return idg_degrid_host(plan, h_grid, d_uvw, d_aterms, d_taper, h_vis, d_workspace, workspace_bytes, stream);
+        const size_t per = adder_buffer_bytes(plan);
+        if (!d_workspace || workspace_bytes < size_t(2) * kStagingBuffers * per)
+            return fail(IDG_ERR_WORKSPACE_TOO_SMALL, "idg_degrid_host_splitter needs idg_host_adder_workspace_size() = " +
+                                                         std::to_string(size_t(2) * kStagingBuffers * per) + " bytes");
+        const DeviceCopy *dc = nullptr;
+        if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        std::lock_guard<std::mutex> lock(*dc->pipeline_mu);
+        const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+        const size_t bl_bytes = size_t(plan->nr_timesteps) * plan->nr_channels * 32;
+        const int64_t bl_f2 = int64_t(plan->nr_timesteps) * plan->nr_channels * 4;
+        const int64_t bl_vis = int64_t(plan->nr_timesteps) * plan->nr_channels;
+        const size_t sgb = subgrid_bytes(plan);
+        const int nb = int(std::max<size_t>(kStagingBuffers, std::min(workspace_bytes / (2 * per), plan->groups.size())));
+        char *base = static_cast<char *>(d_workspace) + size_t(nb) * per;   // degrid half
+        const char *what = "";
+        PipeEvents *pe = nullptr;
+        cudaError_t e = pipe_events(dc, d_workspace, nb, &pe);
+        if (e == cudaSuccess) e = host_subgrid_buffers(pe, 2 * nb, size_t(plan->group_items) * sgb);
+        if (e != cudaSuccess) return cuda_fail(e, "idg_degrid_host_splitter: events / host buffers");
+        HostPool pool(host_threads());
+        auto *grid = const_cast<std::complex<float> *>(static_cast<const std::complex<float> *>(h_grid));
+        size_t last = 0;
+        // the host reads h_grid while the caller's earlier work on `stream` may still write it
+        IDG_PIPE(cudaStreamSynchronize(s));
+        for (size_t gi = 0; gi < plan->groups.size(); ++gi) {
+            const WorkGroup &g = plan->groups[gi];
+            const int b = int(gi % nb);
+            char *vbuf = base + size_t(b) * per;
+            auto *sbuf = reinterpret_cast<float2 *>(vbuf + plan->group_bytes);
+            void *hsub = pe->host_subgrids[nb + b];
+            const size_t bytes = size_t(g.b1 - g.b0) * bl_bytes;
+            if (g.i1 > g.i0) {
+                // host splitter: the previous upload from this host buffer must have finished
+                IDG_PIPE(cudaEventSynchronize(pe->h2d[b]));
+                host_add_or_split(plan, pool, g.i0, g.i1, grid, static_cast<std::complex<float> *>(hsub), false);
+                IDG_PIPE(cudaStreamWaitEvent(dc->h2d, pe->kernel_d[b], 0));   // the kernel that last read sbuf
+                IDG_PIPE(cudaMemcpyAsync(sbuf, hsub, size_t(g.i1 - g.i0) * sgb, cudaMemcpyHostToDevice, dc->h2d));
+                IDG_PIPE(cudaEventRecord(pe->h2d[b], dc->h2d));
+                IDG_PIPE(cudaStreamWaitEvent(s, pe->h2d[b], 0));
+            }
+            IDG_PIPE(cudaStreamWaitEvent(s, pe->d2h[b], 0));   // the visibility buffer's previous download
+            IDG_PIPE(zero_dropped(dc, vbuf, int64_t(g.b0) * bl_vis, g.r0, g.r1, s));
+            if (g.i1 > g.i0) {
+                idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper,
+                                              reinterpret_cast<float2 *>(vbuf) - int64_t(g.b0) * bl_f2, nullptr);
+                a.subgrids = sbuf;
+                a.order = dc->iota + g.i0;
+                a.nr_items = g.i1 - g.i0;
+                IDG_PIPE(idg::launch_degridder(a, s));
+            }
+            IDG_PIPE(cudaEventRecord(pe->kernel_d[b], s));
+            IDG_PIPE(cudaStreamWaitEvent(dc->d2h, pe->kernel_d[b], 0));
+            IDG_PIPE(cudaMemcpyAsync(static_cast<char *>(h_vis) + size_t(g.b0) * bl_bytes, vbuf, bytes,
+                                     cudaMemcpyDeviceToHost, dc->d2h));
+            IDG_PIPE(cudaEventRecord(pe->d2h[b], dc->d2h));
+            last = gi;
+        }
+        for (int b = 0; b < nb && size_t(b) <= last; ++b) IDG_PIPE(cudaStreamWaitEvent(s, pe->d2h[b], 0));
+        return IDG_OK;
+    pipe_error:
+        return cuda_fail(e, std::string("idg_degrid_host_splitter: ") + what);
+    } catch (const std::exception &ex) {
+        return fail(IDG_ERR_INVALID_ARG, ex.what());
+    }
+}
+#undef IDG_PIPE
+
+}  // extern "C"
+
+extern "C" {
 
 static idg_status rho_benchmark(int32_t rho, int32_t iterations, idg_stream stream, double *ops_per_second,
                                 double *seconds, bool packed) {

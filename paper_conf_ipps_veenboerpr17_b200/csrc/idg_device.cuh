@@ -184,6 +184,10 @@ __device__ __forceinline__ void gridder_epilogue(const KernelArgs &a, const Item
             idx += step;
             idx -= (idx >= NS) ? NS : 0;
         }
+        if (a.subgrids) {   // host adder: store into the item's slot of the subgrid buffer
+            a.subgrids[int64_t(blockIdx.x) * 4 * NPIX + o] = sum;
+            continue;
+        }
         float2 *dst = a.grid + ((int64_t(md.z) * 4 + pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx;
         red_add(dst, sum);
     }
@@ -200,7 +204,8 @@ __device__ __forceinline__ void degridder_split_columns(const KernelArgs &a, con
     const idg_metadata &md = s.md;
     for (int o = threadIdx.x; o < 4 * NPIX; o += nt) {
         const int pol = o / NPIX, rem = o - pol * NPIX, ky = rem / NS, kx = rem - ky * NS;
-        sub_s[o] = a.grid[((int64_t(md.z) * 4 + pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx];
+        sub_s[o] = a.subgrids ? a.subgrids[int64_t(blockIdx.x) * 4 * NPIX + o]   // host splitter
+                              : a.grid[((int64_t(md.z) * 4 + pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx];
     }
     init_twiddles<NS>(tw, +1.0f);
     __syncthreads();

@@ -46,6 +46,9 @@ struct KernelArgs {
     const float *taper;          // [N~][N~]
     float2 *vis;                 // [nbl][T][C][4]  (const for gridding)
     float2 *grid;                // [4][N][N]       (const for degridding)
+    float2 *subgrids;            // nullptr, or [nr_items][4][N~][N~] in launch order: the gridders store their
+                                 // transformed subgrids here instead of adding them to `grid`, the
+                                 // degridders read their split subgrids from here (host adder / splitter)
     int32_t max_channels_in_item;
     int32_t max_timesteps_in_item;
     int32_t channel_gcd;         // gcd of all items' channel counts

@@ -220,6 +220,13 @@ __device__ __forceinline__ void gridder_epilogue_tc(const KernelArgs &a, const I
     });
     __syncthreads();
     // a4 columns + a5: G[pol][ky][kx] = sum_y T[pol][y][kx] F[y][ky], added to the grid
+    if (a.subgrids) {   // host adder: the transformed subgrid goes to its slot of the subgrid buffer
+        float2 *sp = a.subgrids + int64_t(blockIdx.x) * 4 * NPIX;
+        dft_pass_tc<NS, WARPS>(tmp_s, NS, 1, tab, 1.0f, 32.0f / sc, [&](int pol, int kx, int ky, float2 v) {
+            sp[(pol * NS + ky) * NS + kx] = v;
+        });
+        return;
+    }
     const int64_t gs = a.grid_size;
     float2 *gp = a.grid + (int64_t(md.z) * 4 * gs + md.y) * gs + md.x;
     dft_pass_tc<NS, WARPS>(tmp_s, NS, 1, tab, 1.0f, 32.0f / sc, [&](int pol, int kx, int ky, float2 v) {
@@ -239,8 +246,10 @@ __device__ __forceinline__ void degridder_prologue_tc(const KernelArgs &a, const
     constexpr int NT = WARPS * 32;
     constexpr int PER = (4 * NPIX + NT - 1) / NT;
     const idg_metadata &md = s.md;
-    const int64_t gs = a.grid_size;
-    const float2 *gp = a.grid + (int64_t(md.z) * 4 * gs + md.y) * gs + md.x;
+    // a6 reads the item's window of the grid, or (host splitter) its slot of the subgrid buffer
+    const int64_t gs = a.subgrids ? NS : a.grid_size;
+    const float2 *gp = a.subgrids ? a.subgrids + int64_t(blockIdx.x) * 4 * NPIX
+                                  : a.grid + (int64_t(md.z) * 4 * gs + md.y) * gs + md.x;
     float2 v[PER];
 #pragma unroll
     for (int i = 0; i < PER; ++i) {   // a6: all loads in flight before any use
@@ -912,7 +921,13 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 // 1..3 by complex products (fp32, on the FMA pipe) before the operand split.  Exact in exact
 // arithmetic; the rounding is that of up to three extra complex products per phasor.
 // ------------------------------------------------------------------------------------------------
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4>
+// SCH (R = 8, 16): issue schedule of the k-block loop.  0: per tile, its rows' rotation + split, then its
+// three products.  2: two independent rotation chains (rows 0..R/2-1 from row 0, rows R/2..R-1 from row
+// R/2, which gets its own sincos) advanced in alternation: half the dependent-chain length for one more
+// sincos pair per k-block (measured: N~ = 32 SKA 2140 -> 2186 MVis/s, predict +0.5%; N~ = 24 LOFAR -3.7%,
+// so it is the default for N~ = 32 only).  A one-tile software pipeline of the HMMAs (tried as SCH = 1)
+// compiles to the same SASS as 0: ptxas already spaces the HMMAs 5-12 instructions apart.
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int SCH = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int NKB = NPIX / 8;
@@ -1002,6 +1017,37 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                 for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
 #pragma unroll
                 for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
+            } else if constexpr (SCH == 2) {
+                // R = 8, 16, two rotation chains: tiles i (rows 2i, 2i+1) and i + NTL/2 (rows R/2 + 2i, ...)
+                constexpr int H = NTL / 2;
+                const f2p ph8 = fma2(dup(float(R / 2)), pk(e.x, e.y), pk(p.x, p.y));
+                const float2 p8 = unpk(ph8);
+                float s8a, c8a, s8b, c8b;
+                __sincosf(p8.x, &s8a, &c8a);
+                __sincosf(p8.y, &s8b, &c8b);
+                f2p C2 = pk(c8a, c8b), S2 = pk(s8a, s8b);
+#pragma unroll
+                for (int i = 0; i < H; ++i) {
+                    uint32_t ah[4], al[4], bh[4], bl[4];
+#pragma unroll
+                    for (int h2 = 0; h2 < 2; ++h2) {
+                        if (i > 0 || h2 > 0) {
+                            const f2p Cn = fma2(C, EC, mul2(S, NES));
+                            S = fma2(C, ES, mul2(S, EC));
+                            C = Cn;
+                            const f2p Cm = fma2(C2, EC, mul2(S2, NES));
+                            S2 = fma2(C2, ES, mul2(S2, EC));
+                            C2 = Cm;
+                        }
+                        const float2 cc = unpk(C), ss = unpk(S), cc2 = unpk(C2), ss2 = unpk(S2);
+                        split_phasor(cc.x, ss.x, ah[h2], al[h2]);
+                        split_phasor(cc.y, ss.y, ah[2 + h2], al[2 + h2]);
+                        split_phasor(cc2.x, ss2.x, bh[h2], bl[h2]);
+                        split_phasor(cc2.y, ss2.y, bh[2 + h2], bl[2 + h2]);
+                    }
+                    mma3(acc[i], ah, al, bf);
+                    mma3(acc[i + H], bh, bl, bf);
+                }
             } else {
                 // R = 8, 16: each tile's three products issued as soon as its two rows are split
 #pragma unroll
@@ -1126,9 +1172,9 @@ template <int NS, int WARPS, int MT, int MINB>
 cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
     return launch_tc(degridder_tc_kernel<NS, WARPS, MT, MINB>, "degridder", smem_degridder_tc<NS>(a), WARPS * 32, a, st);
 }
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int SCH = 0>
 cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
-    return launch_tc(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R>, "degridder", smem_degridder_tc<NS>(a),
+    return launch_tc(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R, SCH>, "degridder", smem_degridder_tc<NS>(a),
                      WARPS * 32, a, st);
 }
 
@@ -1160,6 +1206,9 @@ const Variant kTcGridder[] = {
 #define TDROTC(NS, W, MB, U, CPT, R, TAG) \
     {NS, CPT, kTensor, 1, TAG "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, R>, CPT, smem_degridder_tc<NS>}
+#define TDROTX(NS, W, MB, U, CPT, R, SCH) \
+    {NS, CPT, kTensor, 1, "degridder_rot16s" #SCH "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, R, SCH>, CPT, smem_degridder_tc<NS>}
 #define TDROT(NS, W, MB, U) \
     {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>, 0, \
      smem_degridder_tc<NS>}
@@ -1167,8 +1216,8 @@ const Variant kTcGridder[] = {
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>, 0, \
      smem_degridder_tc<NS>}
 const Variant kTcDegridder[] = {
-    TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"),
-    TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
+    TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 1, 32, 16, 2),
+    TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
     TDROTC(24, 8, 2, 1, 8, 8, "degridder_rot8"), TDROTC(32, 16, 2, 1, 8, 8, "degridder_rot8"),
     TDROTC(16, 8, 2, 1, 8, 8, "degridder_rot8"),
@@ -1176,8 +1225,11 @@ const Variant kTcDegridder[] = {
     TDROTC(24, 8, 4, 1, 4, 4, "degridder_rot"), TDROTC(32, 16, 2, 1, 4, 4, "degridder_rot"),
     TDROTC(16, 8, 4, 1, 4, 4, "degridder_rot"),
     TD(24, 8, 2, 4), TD(32, 8, 4, 2), TD(16, 8, 4, 2),
+    // the single-chain N~ = 32 kernels (selected by name only)
+    TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"),
 };
 #undef TDROTC
+#undef TDROTX
 #undef TDROT
 #undef TD
 

@@ -89,7 +89,9 @@ __global__ void __launch_bounds__(kRhoThreads) rho_kernel<0>(float *out, int ite
 }
 
 // Packed form: U unit pairs per thread; per pair and iteration one FFMA2 forms both arguments, two
-// __sincosf, then rho-1 FFMA2 accumulate (alternating cos / sin pairs) into 8 packed accumulators.
+// __sincosf, then rho-1 FFMA2 accumulate (alternating cos / sin pairs) into 8 packed accumulators.  The
+// accumulate coefficient is a kernel parameter (a uniform register), so an FFMA2 reads two 64-bit
+// register pairs: with three (scripts/rho_forms_probe.cu, B200) rho = 17 reaches 55 TOps/s instead of 61.
 using u64 = unsigned long long;
 __device__ __forceinline__ u64 pk2(float lo, float hi) {
     u64 r;
@@ -110,12 +112,10 @@ __device__ __forceinline__ u64 ffma2(u64 a, u64 b, u64 c) {
 constexpr int kRhoPairs = 4;   // unit pairs per thread (8 units)
 
 template <int RHO>
-__global__ void __launch_bounds__(kRhoThreads) rho_kernel_x2(float *out, int iterations) {
+__global__ void __launch_bounds__(kRhoThreads) rho_kernel_x2(float *out, int iterations, u64 coef) {
     constexpr int U = kRhoPairs;
     const int tid = blockIdx.x * blockDim.x + threadIdx.x;
-    u64 sn[U], cs[U], acc[U][8], coef[8];
-#pragma unroll
-    for (int j = 0; j < 8; ++j) coef[j] = pk2(0.25f + 0.01f * float((tid + j) & 7), 0.26f + 0.01f * float((tid + j) & 7));
+    u64 sn[U], cs[U], acc[U][8];
 #pragma unroll
     for (int k = 0; k < U; ++k) {
         sn[k] = pk2(0.1f * float(k) + 1e-6f * float(tid & 1023), 0.05f * float(k) + 1e-6f * float(tid & 511));
@@ -136,7 +136,7 @@ __global__ void __launch_bounds__(kRhoThreads) rho_kernel_x2(float *out, int ite
             cs[k] = pk2(c0, c1);
 #pragma unroll
             for (int j = 0; j < RHO - 1; ++j)                  // FMAs #2 .. #rho of both units
-                acc[k][j & 7] = ffma2(coef[(j >> 3) & 7], (j & 1) ? sn[k] : cs[k], acc[k][j & 7]);
+                acc[k][j & 7] = ffma2(coef, (j & 1) ? sn[k] : cs[k], acc[k][j & 7]);
         }
     }
     float sum = 0.0f;
@@ -153,8 +153,8 @@ __global__ void __launch_bounds__(kRhoThreads) rho_kernel_x2(float *out, int ite
     out[tid] = sum;
 }
 
-template <typename K>
-cudaError_t run_kernel(K kernel, int iterations, float *out, cudaStream_t s, int *blocks) {
+template <typename K, typename... Extra>
+cudaError_t run_kernel(K kernel, int iterations, float *out, cudaStream_t s, int *blocks, Extra... extra) {
     int per_sm = 0, dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceProp prop;
@@ -162,7 +162,7 @@ cudaError_t run_kernel(K kernel, int iterations, float *out, cudaStream_t s, int
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, kRhoThreads, 0);
     *blocks = prop.multiProcessorCount * (per_sm > 0 ? per_sm : 1) * 4;  // 4 full waves
     LaunchScope scope("rho_benchmark", s);
-    kernel<<<*blocks, kRhoThreads, 0, s>>>(out, iterations);
+    kernel<<<*blocks, kRhoThreads, 0, s>>>(out, iterations, extra...);
     return cudaGetLastError();
 }
 
@@ -170,7 +170,7 @@ template <int RHO>
 cudaError_t run(int iterations, float *out, cudaStream_t s, int *blocks, bool packed, int *units) {
     if (packed && RHO > 0) {
         *units = 2 * kRhoPairs;
-        return run_kernel(rho_kernel_x2<RHO>, iterations, out, s, blocks);
+        return run_kernel(rho_kernel_x2<RHO>, iterations, out, s, blocks, 0x3e8a00003e800000ull);  // (0.25, 0.27)
     }
     *units = RHO == 0 ? 8 : kRhoUnits;
     return run_kernel(rho_kernel<RHO>, iterations, out, s, blocks);

@@ -48,6 +48,7 @@ EXPORTED = ["idg_plan_create", "idg_plan_destroy", "idg_plan_nr_subgrids", "idg_
             "idg_rho_benchmark_scalar",
             "idg_profiling_enable", "idg_profiling_reset", "idg_profiling_read", "idg_launch_count",
             "idg_kernel_variants", "idg_host_workspace_size", "idg_grid_host", "idg_degrid_host",
+            "idg_host_adder_workspace_size", "idg_grid_host_adder", "idg_degrid_host_splitter",
             "idg_status_string", "idg_last_error", "idg_last_variant"]
 
 
@@ -73,6 +74,9 @@ def lib() -> ctypes.CDLL:
     L.idg_host_workspace_size.argtypes = [P, ctypes.POINTER(sz)]
     L.idg_grid_host.argtypes = [P, P, P, P, P, P, P, sz, P]
     L.idg_degrid_host.argtypes = [P, P, P, P, P, P, P, sz, P]
+    L.idg_host_adder_workspace_size.argtypes = [P, ctypes.POINTER(sz)]
+    L.idg_grid_host_adder.argtypes = [P, P, P, P, P, P, P, sz, P]
+    L.idg_degrid_host_splitter.argtypes = [P, P, P, P, P, P, P, sz, P]
     for f in ("idg_rho_benchmark", "idg_rho_benchmark_scalar"):
         getattr(L, f).argtypes = [i32, i32, P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
     L.idg_profiling_enable.argtypes = [i32]
@@ -176,6 +180,11 @@ class Plan:
         _check(lib().idg_workspace_size(self._h, ctypes.byref(b)), "idg_workspace_size")
         return int(b.value)
 
+    def host_adder_workspace_size(self) -> int:
+        b = ctypes.c_size_t()
+        _check(lib().idg_host_adder_workspace_size(self._h, ctypes.byref(b)), "idg_host_adder_workspace_size")
+        return int(b.value)
+
     def host_workspace_size(self) -> int:
         b = ctypes.c_size_t()
         _check(lib().idg_host_workspace_size(self._h, ctypes.byref(b)), "idg_host_workspace_size")
@@ -256,14 +265,19 @@ def _host(t, dtype, shape, name):
     return ctypes.c_void_p(t.data_ptr())
 
 
-def workspace(plan: Plan, device=None, full: bool = False):
+def workspace(plan: Plan, device=None, full: bool = False, max_buffers: int = 0):
     """A device workspace for the host-streamed calls: the minimum (idg_host_workspace_size, three
-    staging buffers per direction) or, with full=True, one staging buffer per work group and direction
-    (2 x the visibility bytes) so consecutive grid/degrid calls overlap completely."""
+    staging buffers per direction); with full=True one staging buffer per work group and direction
+    (2 x the visibility bytes) so consecutive grid/degrid calls overlap completely; with max_buffers=k
+    up to k staging buffers per direction (no more than one per work group)."""
     import torch
     n = plan.host_workspace_size()
+    per_buffer = n // 6                        # idg_host_workspace_size = 2 directions x 3 buffers
+    all_groups = 2 * plan.nr_baselines * plan.nr_timesteps * plan.nr_channels * 32 + (64 << 20)
     if full:
-        n = max(n, 2 * plan.nr_baselines * plan.nr_timesteps * plan.nr_channels * 32 + (64 << 20))
+        n = max(n, all_groups)
+    elif max_buffers > 3:
+        n = max(n, min(all_groups, 2 * max_buffers * per_buffer))
     return torch.empty(max(1, n), dtype=torch.uint8, device=device or "cuda")
 
 
@@ -296,6 +310,39 @@ def degrid_host(plan: Plan, grid_in, uvw, aterms, taper, vis_host_out, ws, strea
     with _one_device(grid_in, uvw, aterms, taper, ws):
         _check(lib().idg_degrid_host(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(),
                                      _stream(stream)), "idg_degrid_host")
+    return vis_host_out
+
+
+def adder_workspace(plan: Plan, device=None, buffers: int = 3):
+    """A device workspace for the host adder / splitter calls: `buffers` (>= 3) staging buffers per direction."""
+    import torch
+    n = plan.host_adder_workspace_size() * max(3, int(buffers)) // 3
+    return torch.empty(max(1, n), dtype=torch.uint8, device=device or "cuda")
+
+
+def grid_host_adder(plan: Plan, vis_host, uvw, aterms, taper, grid_host_out, ws, stream=None):
+    """idg_grid_host_adder: visibilities and the grid in HOST memory; subgrids added on the host."""
+    sh = _shapes(plan)
+    args = [_host(vis_host, *sh["vis"], "vis_host"), _dev(uvw, *sh["uvw"], "uvw"),
+            _dev(aterms, *sh["aterms"], "aterms"), _dev(taper, *sh["taper"], "taper"),
+            _host(grid_host_out, *sh["grid"], "grid_host")]
+    _workspace_ok(ws)
+    with _one_device(uvw, aterms, taper, ws):
+        _check(lib().idg_grid_host_adder(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(),
+                                         _stream(stream)), "idg_grid_host_adder")
+    return grid_host_out
+
+
+def degrid_host_splitter(plan: Plan, grid_host, uvw, aterms, taper, vis_host_out, ws, stream=None):
+    """idg_degrid_host_splitter: the model grid in HOST memory, subgrids split on the host."""
+    sh = _shapes(plan)
+    args = [_host(grid_host, *sh["grid"], "grid_host"), _dev(uvw, *sh["uvw"], "uvw"),
+            _dev(aterms, *sh["aterms"], "aterms"), _dev(taper, *sh["taper"], "taper"),
+            _host(vis_host_out, *sh["vis"], "vis_host_out")]
+    _workspace_ok(ws)
+    with _one_device(uvw, aterms, taper, ws):
+        _check(lib().idg_degrid_host_splitter(plan.handle, *args, ctypes.c_void_p(ws.data_ptr()), ws.numel(),
+                                              _stream(stream)), "idg_degrid_host_splitter")
     return vis_host_out
 
 

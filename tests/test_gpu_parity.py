@@ -217,6 +217,46 @@ def test_host_streamed_calls(name, kw, chunk, drop, monkeypatch):
     assert torch.equal(v_host, v_dev.cpu())
 
 
+@pytest.mark.parametrize("name,kw,chunk,drop", [("small_dde", {}, 50000, False),
+                                                ("small_dde", dict(w_planes=3), 60000, False),
+                                                ("lofar", dict(T=640, nr_stations=6), 300000, False),
+                                                ("ska", dict(T=256, nr_stations=4), 2000000, False),
+                                                ("small_dde", {}, 50000, True)])
+def test_host_adder_and_splitter(name, kw, chunk, drop, monkeypatch):
+    """The grid in host memory (option 2): subgrids stream to / from the host and host threads add
+    them into / split them out of the grid.  Against the oracle, and degridding bit-identical to the
+    device-resident call (same kernels, same subgrids)."""
+    import dataclasses
+    monkeypatch.setenv("IDG_HOST_CHUNK_BYTES", str(chunk))     # several work groups
+    monkeypatch.setenv("IDG_HOST_THREADS", "5")                # rows interleaved over an odd thread count
+    obs = idgsynth.make_observation(name, **kw)
+    if drop:
+        obs = dataclasses.replace(obs, image_size=obs.image_size * 6)
+    vis, aterms, tap = _inputs(obs, None, "asymmetric")
+    items, dropped = oracle.plan(obs)
+    assert (dropped > 0) == drop
+    plan = idg.Plan.from_observation(obs)
+    ws = idg.adder_workspace(plan, buffers=4)
+    uvw, at, tp = _dev(obs.uvw), _dev(aterms), _dev(tap)
+    vis_h = torch.from_numpy(vis).pin_memory()
+    g_host = torch.zeros(oracle.grid_shape(obs), dtype=torch.complex64)
+    idg.grid_host_adder(plan, vis_h, uvw, at, tp, g_host, ws)
+    idg.grid_host_adder(plan, vis_h, uvw, at, tp, g_host, ws)      # accumulates
+    ref = 2 * oracle.grid(obs, items, vis, aterms, tap)
+    err = rel_rms(g_host.numpy(), ref)
+    print(f"host adder {name} {kw}: rel rms {err:.3e}")
+    assert err <= TOL, err
+    G = idgsynth.make_grid(obs)
+    refv = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, G, aterms, tap))
+    v_host = torch.full((obs.nr_baselines, obs.nr_timesteps, obs.nr_channels, 4), complex(3, 3),
+                        dtype=torch.complex64).pin_memory()
+    idg.degrid_host_splitter(plan, torch.from_numpy(G), uvw, at, tp, v_host, ws)
+    torch.cuda.synchronize()
+    assert rel_rms(v_host.numpy(), refv) <= TOL
+    v_dev = gpu_degrid(obs, G, aterms, tap, plan)
+    assert torch.equal(v_host, v_dev.cpu())
+
+
 def test_host_streamed_upload_waits_for_the_callers_stream():
     """A non-blocking device->host copy into vis_h queued on the caller's stream right before
     idg_grid_host (no synchronize in between): the uploads must see the new host data."""
