@@ -35,7 +35,7 @@ import idgsynth  # noqa: E402
 BASELINE = json.load(open(os.path.join(ROOT, "BASELINE.json")))
 METRIC = BASELINE["metric"]
 OPS_PER_PAIR = 36        # 17 FMA (2 ops) + sin + cos per (pixel, visibility) pair
-CONFIG_NAMES = {"tiny": 0, "lofar": 1, "lofar_dde": 2, "ska": 3, "predict": 4}
+CONFIG_NAMES = {"tiny": 0, "lofar": 1, "lofar_dde": 2, "ska": 3, "predict": 4, "lofar_short": 1}
 
 
 def log(*a):
@@ -116,7 +116,9 @@ def dist_env():
 
 def workload_description(name):
     obs_cfg = idgsynth.CONFIGS[name]
-    return (f"{BASELINE['configs'][CONFIG_NAMES[name]]} | synthetic: {obs_cfg['nr_stations']} stations, "
+    short = (" [short-item variant: dt=8 s over 18 h, N=8192 -- not a BASELINE config]" if name == "lofar_short"
+             else "")
+    return (f"{BASELINE['configs'][CONFIG_NAMES[name]]}{short} | synthetic: {obs_cfg['nr_stations']} stations, "
             f"T={obs_cfg['T']}, C={obs_cfg['C']}, N~={obs_cfg['Ns']}, N={obs_cfg['N']}, K={obs_cfg['K']}, "
             f"T~max={obs_cfg['Tmax']}, A-terms={obs_cfg['aterms']} (slots of {obs_cfg['slot']})")
 
@@ -205,7 +207,7 @@ def run_reference(args):
 # A step per config: SKA-, LOFAR-shaped and tiny sets grid then degrid (the imaging cycle's two kernels,
 # P:45-47); the predict sweep (configs[4]) degrids only, from a model grid broadcast by rank 0.
 STEP_KIND = {"tiny": "grid+degrid", "lofar": "grid+degrid", "lofar_dde": "grid+degrid", "ska": "grid+degrid",
-             "predict": "degrid"}
+             "predict": "degrid", "lofar_short": "grid+degrid"}
 # e2e: the SKA-shaped set streams from the host as time chunks ("8 time chunks of 1024")
 E2E_TIME_CHUNK = {"ska": 1024}
 TENSOR_FLOPS_PER_PAIR = 96   # split-f16 contraction: 3 products x 16 real MACs x 2 flops per pair
@@ -422,10 +424,31 @@ def run_ours(args):
         energy["per_kernel"] = per
         energy["paper_context"] = "GTX 1080: 32 / 23 GFlops/W gridder / degridder (P:306; paper-ops: 17 FMA + sincos)"
 
+    # ---- one full imaging cycle, timed per stage (Fig. 9: "runtime is dominated by the gridder and
+    # degridder kernels (more than 93%)"); grid+degrid configs, one GPU
+    cycle = None
+    if kind == "grid+degrid" and world == 1 and not args.no_imaging_cycle:
+        from paper_conf_ipps_veenboerpr17_b200 import imaging
+        N = obs.grid_size
+        tap_img = torch.ones((N, N), dtype=torch.float32, device=dev)   # the taper function on the image grid
+        for _ in range(2):   # warm-up (cuFFT plans), then the timed cycle
+            stages = imaging.imaging_cycle(plan, vis_d, uvw_d, at_d, tp_d, tap_img, out_d, stream=stream)
+        tot = stages["total_ms"]
+        cycle = {"ms": stages, "share": {k: v / tot for k, v in stages.items() if k != "total_ms"},
+                 "kernels_share": (stages["grid"] + stages["degrid"]) / tot,
+                 "note": "grid / degrid are the fused kernels (subgrid FFT, adder / splitter, A-term and taper "
+                         "inside); ifft / fft are cuFFT on the 4 x N^2 complex64 grid; the dirty image stands in "
+                         "for the deconvolved model" + ("; residual skipped (predictions written in place)"
+                                                        if inplace else ""),
+                 "paper_context": "P:258: gridder + degridder > 93% of the cycle on Haswell / Fiji / Pascal"}
+        del tap_img
+
     # ---- e2e: host buffers through the public API ------------------------------------------------
-    e2e = None if args.no_e2e else run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream,
-                                           world, rank, nvis_total, vis_d, out_d, grid_d, sharded, barrier, inplace)
+    bufs = {"vis": vis_d, "out": out_d}
     del vis_d, out_d
+    e2e = None if args.no_e2e else run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream,
+                                           world, rank, nvis_total, bufs, grid_d, sharded, barrier, inplace)
+    bufs.clear()
 
     # ---- roofline ---------------------------------------------------------------------------------
     def best(rho, iters, scalar=False):
@@ -503,12 +526,17 @@ def run_ours(args):
                                  "accumulation; sincos of one channel group / row per pixel, the other channels by "
                                  "exact rotation (uniform channels)",
                    "subgrids_rank0": st["nr_subgrids"], "pairs_rank0": pairs,
+                   "items_timesteps": {"mean": float(md["nr_timesteps"].mean()) if len(md) else 0.0,
+                                       "median": float(np.median(md["nr_timesteps"])) if len(md) else 0.0,
+                                       "hist_bins_of_16": (np.bincount(np.minimum(md["nr_timesteps"], 128) // 16,
+                                                                       minlength=9) / max(1, len(md))).round(4).tolist()},
                    "parallelism": f"baseline shards x{world}" + (" + NCCL reduce/broadcast" if world > 1 else ""),
                    "l2": f"inputs larger than L2 (visibilities {vis_bytes / 1e9:.1f} GB/step)",
                    "degrid_in_place": inplace},
         "grid_mvis_s": per_kernel.get("gridder", {}).get("mvis_s"),
         "degrid_mvis_s": per_kernel.get("degridder", {}).get("mvis_s"),
         "plan_s": plan_s, "clocks": clocks.summary(), "energy": energy, "e2e": e2e, "gpu_launches": gpu_launches,
+        "imaging_cycle": cycle,
         "roofline": roofline, "kernels": per_kernel, "rho_sweep_TOps_s": rho_sweep or None,
         "cpu_baseline": cpu,
     }
@@ -518,14 +546,15 @@ def run_ours(args):
     return 0
 
 
-def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, world, rank, nvis_total, vis_d,
-            out_d, grid_d, sharded, barrier, inplace):
+def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, world, rank, nvis_total, bufs,
+            grid_d, sharded, barrier, inplace):
     """The metric end to end through the public host-streamed calls (idg_grid_host / idg_degrid_host, the
     paper's triple-buffered work groups): every step uploads its inputs (visibilities, uvw,
     A-terms; the model grid for predict) from page-locked host memory and downloads the predictions.
     The SKA-shaped set streams as time chunks of 1024 (one plan per chunk)."""
     import torch
     import torch.distributed as dist
+    vis_d, out_d = bufs["vis"], bufs["out"]
     try:
         import psutil
         host_avail = psutil.virtual_memory().available
@@ -592,6 +621,7 @@ def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, wo
         nb_chk = min(64, nbl)
         chk_ref = out_d[:nb_chk].cpu()
     del vis_d, out_d
+    bufs.clear()                 # the device-resident arrays are freed here (the caller holds no reference)
     torch.cuda.empty_cache()
     # one workspace, grid, uvw and A-term buffer per stream: a workspace serves one in-flight call.  Steps
     # rotate over NS streams: a host-streamed call starts its uploads after the work queued before it on its
@@ -644,9 +674,14 @@ def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, wo
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     check = None
     out_last = out_h
-    if kind == "grid+degrid" and not rotating and world == 1:
-        # whole-data check: degrid = grid^H, so <vis, degrid(grid(vis))> = ||grid(vis)||^2 (adjoint identity)
+    if kind == "grid+degrid" and not rotating:
+        # whole-data check: degrid = grid^H, so <vis, degrid(grid(vis))> = ||grid(vis)||^2 (adjoint identity;
+        # with N ranks the left side sums over the shards and the grid is the reduced + broadcast one)
         lhs = vdot_chunked(in_h, out_last, dev)
+        if world > 1:
+            t2 = torch.tensor([lhs.real, lhs.imag], dtype=torch.float64, device=dev)
+            dist.all_reduce(t2)
+            lhs = complex(float(t2[0]), float(t2[1]))
         g = grids[(ksteps - 1) % NS]
         rhs = float(torch.linalg.vector_norm(g.view(torch.float32).to(torch.float64)) ** 2)
         check = {"adjoint_identity_rel_err": abs(lhs - rhs) / abs(rhs)}
@@ -686,6 +721,7 @@ def main():
     ap.add_argument("--rho-iterations", type=int, default=16384)
     ap.add_argument("--no-rho-sweep", action="store_true")
     ap.add_argument("--no-kernel-energy", action="store_true")
+    ap.add_argument("--no-imaging-cycle", action="store_true")
     ap.add_argument("--energy-launches", type=int, default=5)
     ap.add_argument("--timesteps", type=int, default=0,
                     help="tuning only: override the config's T (the line then names the reduced workload)")

@@ -188,6 +188,11 @@ CONFIGS = {
     "small_dde": dict(layout="lofar", nr_stations=8, lat=52.91, dec=60.0, C=4, f0=150e6, df=195.3e3, T=96,
                       dt=20.0, Ns=16, N=256, K=5, Tmax=24, slot=40, aterms="random", seed=1010,
                       w_offset="half_median"),
+    # short-item stress variant of configs[1] (not a BASELINE config): 8 s integration over 18 h on an 8192^2
+    # grid, so the uv tracks cross subgrids ~16x faster per time step -- mean T~ 46, median 24 (P:254:
+    # "performance is data dependent")
+    "lofar_short": dict(layout="lofar", nr_stations=44, lat=52.91, dec=60.0, C=16, f0=150e6, df=12.207e3, T=8192,
+                        dt=8.0, Ns=24, N=8192, K=7, Tmax=128, slot=256, aterms="identity", seed=1006),
     "ska": dict(layout="spiral", nr_stations=150, lat=-26.82, dec=-30.0, C=32, f0=140e6, df=24.414e3, T=8192,
                 dt=1.0, Ns=32, N=8192, K=9, Tmax=128, slot=256, aterms="identity", seed=1004),
     "predict": dict(layout="spiral_ext", nr_stations=512, lat=-26.82, dec=-30.0, C=16, f0=140e6, df=24.414e3,

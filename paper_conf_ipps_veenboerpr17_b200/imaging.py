@@ -90,3 +90,67 @@ def find_peak(image, pol: int = 0):
     idx = int(torch.argmax(re))
     y, x = divmod(idx, re.shape[-1])
     return float(re[y, x]), y, x
+
+
+def imaging_cycle(plan: idg.Plan, vis, uvw, aterms, taper, taper_image, vis_out, stream=None, residual=True):
+    """One full imaging cycle (Fig. 2) in production precision (complex64 throughout), timed per
+    stage with CUDA events on `stream` -- the analogue of the paper's runtime breakdown (Fig. 9):
+
+      grid      zero the uv-grid(s) + idg_grid (gridder, A-term/taper, subgrid FFT, adder: one fused kernel)
+      ifft      centred inverse FFT of every polarisation / W-plane (cuFFT via torch.fft)
+      image     taper + w0 corrections -> dirty image (elementwise)
+      model     the dirty image stands in for the deconvolved model (deconvolution is out of scope):
+                corrections + centred FFT back to the model grid(s)
+      degrid    idg_degrid (splitter, subgrid iFFT, taper/A-term, degridder: one fused kernel)
+      residual  vis - predicted (elementwise; skipped when vis_out aliases vis)
+
+    Returns {stage: ms} plus 'total_ms'.  vis_out receives the residual (the unnormalised predictions, x N~^2,
+    when it aliases vis)."""
+    s = torch.cuda.current_stream(vis.device) if stream is None else stream
+    N = plan.grid_size
+    nz = plan.nr_w_planes
+    shape = (4, N, N) if nz == 1 else (nz, 4, N, N)
+    ev = {}
+
+    def mark(name):
+        e = torch.cuda.Event(enable_timing=True)
+        e.record(s)
+        ev[name] = e
+
+    with torch.cuda.stream(s):
+        _, _, n = image_lmn(plan, vis.device)
+        n = n.to(torch.float32)
+        w0s = _plane_w0(plan)
+        tap = taper_image.to(torch.float32)
+        nvis = max(1, plan.stats()["nr_vis_assigned"])
+        g = torch.empty(shape, dtype=torch.complex64, device=vis.device)
+        mark("start")
+        g.zero_()
+        idg.grid(plan, vis, uvw, aterms, taper, g, stream=s)
+        mark("grid")
+        planes = g.reshape(nz, 4, N, N)
+        img_planes = _centred_ifft2(planes)
+        mark("ifft")
+        img = torch.zeros((4, N, N), dtype=torch.complex64, device=vis.device)
+        for z, w0 in enumerate(w0s):
+            img += img_planes[z] * torch.exp(2j * math.pi * w0 * n) if w0 != 0.0 else img_planes[z]
+        img /= tap * (nvis * plan.subgrid_size ** 2)
+        mark("image")
+        base = img / tap
+        model = torch.stack([base * torch.exp(-2j * math.pi * w0 * n) if w0 != 0.0 else base for w0 in w0s])
+        G = _centred_fft2(model)
+        G = G[0] if nz == 1 else G
+        mark("model")
+        idg.degrid(plan, G.contiguous(), uvw, aterms, taper, vis_out, stream=s)
+        mark("degrid")
+        if residual and vis_out.data_ptr() != vis.data_ptr():
+            vis_out.sub_(vis).neg_()          # residual = vis - predicted
+        mark("residual")
+    ev["residual"].synchronize()
+    names = ["grid", "ifft", "image", "model", "degrid", "residual"]
+    out, prev = {}, "start"
+    for k in names:
+        out[k] = ev[prev].elapsed_time(ev[k])
+        prev = k
+    out["total_ms"] = ev["start"].elapsed_time(ev["residual"])
+    return out

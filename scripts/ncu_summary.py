@@ -80,11 +80,43 @@ def summarize(rep):
             bk = max(pipes, key=pipes.get)
             rec["binding pipe"] = f"{bk} {pipes[bk]:.1f}%"
             rec["_pipes"] = pipes
+        ph = loop_share(rep, name)
+        if ph is not None:
+            rec["inner-loop share of stall samples"] = f"{100 * ph:.1f}% (per-item prologue / epilogue: {100 * (1 - ph):.1f}%)"
+            rec["_loop_share"] = ph
         ia = d.get("smsp__issue_active.avg.pct_of_peak_sustained_active")
         if ia:
             rec["_issue"] = float(ia[1].replace(",", ""))
         res.append(rec)
     return res
+
+
+def loop_share(rep, kernel_name):
+    """Share of the warp-stall samples in the kernel's inner loop: SASS instructions executed at least 5% as
+    often as the most executed one (per-item code -- setup, A-term / taper, subgrid DFT, adder / splitter,
+    stores -- runs ~100x less often).  None without a source page."""
+    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                         capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    try:
+        hi = next(i for i, r in enumerate(rows) if "# Samples" in r and "Instructions Executed" in r)
+    except StopIteration:
+        return None
+    hdr = rows[hi]
+    si, ei = hdr.index("# Samples"), hdr.index("Instructions Executed")
+    data = []
+    for r in rows[hi + 1:]:
+        if len(r) <= max(si, ei):
+            continue
+        try:
+            data.append((float(r[si]), float(r[ei])))
+        except ValueError:
+            continue
+    if not data:
+        return None
+    mx = max(e for _, e in data)
+    tot = sum(smp for smp, _ in data)
+    return sum(smp for smp, e in data if e >= 0.05 * mx) / tot if tot else None
 
 
 def launches(path):
@@ -133,6 +165,7 @@ def main():
                 p = rec["_pipes"]
                 bk = max(p, key=p.get)
                 ent.update({"binding_pipe": bk, "binding_pipe_frac": p[bk] / 100.0,
+                            "inner_loop_sample_share": rec.get("_loop_share"),
                             "issue_active_frac": rec.get("_issue", 0.0) / 100.0,
                             "pipes_pct_of_peak": dict(sorted(p.items(), key=lambda x: -x[1]))})
             js.setdefault(args.config, {})[short] = ent

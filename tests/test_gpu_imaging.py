@@ -71,3 +71,21 @@ def test_point_sources_image_and_predict(w_planes):
     imaging.predict(plan, model, uvw, at, tp, timg, pred)
     res = vis - pred.cpu().numpy()
     assert np.linalg.norm(res) < 0.75 * np.linalg.norm(vis)
+
+
+def test_imaging_cycle_breakdown():
+    """One timed imaging cycle (Fig. 9 analogue): every stage reports a time, the stages add up to the
+    total, and the residual of a cycle whose model is its own dirty image is the data minus its prediction."""
+    obs = idgsynth.make_observation("lofar", T=256, nr_stations=6)
+    plan = idg.Plan.from_observation(obs)
+    dev = torch.device("cuda")
+    vis = torch.from_numpy(idgsynth.make_visibilities(obs)).to(dev)
+    uvw = torch.from_numpy(obs.uvw).to(dev)
+    at = torch.from_numpy(idgsynth.make_aterms(obs)).to(dev)
+    tp = torch.from_numpy(idgsynth.make_taper(obs.subgrid_size)).to(dev)
+    out = torch.empty_like(vis)
+    t = imaging.imaging_cycle(plan, vis, uvw, at, tp, _taper_image(obs, dev), out)
+    stages = ["grid", "ifft", "image", "model", "degrid", "residual"]
+    assert all(t[k] >= 0 for k in stages) and t["grid"] > 0 and t["degrid"] > 0
+    assert abs(sum(t[k] for k in stages) - t["total_ms"]) < 1e-3 * t["total_ms"] + 1e-3
+    assert torch.isfinite(torch.view_as_real(out)).all()
