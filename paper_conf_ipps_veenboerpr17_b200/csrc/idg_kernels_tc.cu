@@ -504,7 +504,13 @@ __device__ __forceinline__ f2p add2(f2p a, f2p b) {
     return r;
 }
 
-template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB, int TU = 1, int NSM = 0>
+// PKR = 1: the rotation of the groups j > 0 on packed f32x2 pairs.  E^j advances for both pixel rows in one
+// pair of FFMA2 / FMUL2 (4 instead of 8 scalar instructions), and E^j D_j is accumulated as
+// acc += Re(E^j) D_j, acc2 += Im(E^j) D_j on the (re, im) pairs the mma writes (two FFMA2 with a
+// broadcast operand instead of four FFMA per pixel row); i acc2 joins acc once per item (complex
+// multiplication by i is linear).  The same products, half the instructions of the rotation.
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB, int TU = 1, int NSM = 0,
+          int PKR = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const KernelArgs a) {
     constexpr int NT = WARPS * 32;
     constexpr int NPIX = NS * NS;
@@ -557,6 +563,10 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
     }
+    // PKR: the Im(E^j) parts of the rotated groups, per tile and pixel row as (re, im) pairs
+    f2p acc2[PKR ? MT : 1][2];
+#pragma unroll
+    for (int i = 0; i < (PKR ? MT : 1); ++i) acc2[i][0] = acc2[i][1] = 0ull;
     float cur_scale = 0.0f;
 
     const int64_t row = int64_t(a.nr_channels) * 4;  // float2 per timestep
@@ -594,9 +604,14 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
         } else if (bscale < cur_scale) {
             const float f = bscale / cur_scale;  // exact power of two
 #pragma unroll
-            for (int i = 0; i < MT; ++i)
+            for (int i = 0; i < MT; ++i) {
 #pragma unroll
                 for (int j = 0; j < 4; ++j) acc[i][j] *= f;
+                if constexpr (PKR) {
+                    acc2[i][0] = mul2(acc2[i][0], dup(f));
+                    acc2[i][1] = mul2(acc2[i][1], dup(f));
+                }
+            }
             cur_scale = bscale;
         }
         // (4) B fragments of every (timestep, group): column g = 2 pol + im, k-slots q and q+4
@@ -652,6 +667,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
                 } else {
                     float2 er, ei;   // E_t of rows (g, g+8)
                     float pr0 = 1.0f, pi0 = 0.0f, pr1 = 1.0f, pi1 = 0.0f;   // E^j of rows g, g+8
+                    f2p ER = 0, EI = 0, PR = 0, PI = 0;                    // PKR: the same packed over the rows
                     // groups in passes of GP: interleaved mma chains, group 0 into the accumulator,
                     // groups j > 0 fresh and rotated by E^j
 #pragma unroll
@@ -680,12 +696,34 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
                             const f2p C4 = pk(cs[2], cs[3]), S4 = pk(sn[2], sn[3]);
                             const f2p r4 = fma2(C4, C0, mul2(S4, S0));
                             const f2p i4 = sub2(mul2(S4, C0), mul2(C4, S0));
-                            er = unpk(sub2(mul2(r4, r4), mul2(i4, i4)));
-                            ei = unpk(mul2(add2(r4, r4), i4));
+                            ER = sub2(mul2(r4, r4), mul2(i4, i4));
+                            EI = mul2(add2(r4, r4), i4);
+                            er = unpk(ER);
+                            ei = unpk(EI);
                         }
 #pragma unroll
                         for (int j = 0; j < GP; ++j) {
                             if (p0 + j == 0) continue;
+                            if constexpr (PKR) {
+                                if (p0 + j == 1) {
+                                    PR = ER;
+                                    PI = EI;
+                                } else {   // E^j = E^(j-1) E for both rows
+                                    const f2p nr = fma2(PR, ER, mul2(PI, sub2(0ull, EI)));
+                                    PI = fma2(PR, EI, mul2(PI, ER));
+                                    PR = nr;
+                                }
+                                const float2 pr = unpk(PR), pi = unpk(PI);
+                                f2p a0 = pk(acc[i][0], acc[i][1]), a1 = pk(acc[i][2], acc[i][3]);
+                                const f2p d0 = pk(d[j][0], d[j][1]), d1 = pk(d[j][2], d[j][3]);
+                                a0 = fma2(dup(pr.x), d0, a0);               // row g:   Re(E^j) D
+                                a1 = fma2(dup(pr.y), d1, a1);               // row g+8
+                                acc2[i][0] = fma2(dup(pi.x), d0, acc2[i][0]);  // Im(E^j) D
+                                acc2[i][1] = fma2(dup(pi.y), d1, acc2[i][1]);
+                                const float2 u0 = unpk(a0), u1 = unpk(a1);
+                                acc[i][0] = u0.x; acc[i][1] = u0.y; acc[i][2] = u1.x; acc[i][3] = u1.y;
+                                continue;
+                            }
                             if (p0 + j == 1) {
                                 pr0 = er.x; pi0 = ei.x; pr1 = er.y; pi1 = ei.y;
                             } else {
@@ -711,6 +749,10 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
     const float inv = cur_scale > 0.0f ? 1.0f / cur_scale : 1.0f;
 #pragma unroll
     for (int i = 0; i < MT; ++i) {
+        if constexpr (PKR) {   // acc + i acc2
+            const float2 b0 = unpk(acc2[i][0]), b1 = unpk(acc2[i][1]);
+            acc[i][0] -= b0.y; acc[i][1] += b0.x; acc[i][2] -= b1.y; acc[i][3] += b1.x;
+        }
         const int p0 = (warp * MT + i) * 16 + g;
         sub_s[q * NPIX + p0] = make_float2(acc[i][0] * inv, acc[i][1] * inv);
         sub_s[q * NPIX + p0 + 8] = make_float2(acc[i][2] * inv, acc[i][3] * inv);
@@ -1158,9 +1200,9 @@ template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBat
 size_t smem_gridder_rot2(const KernelArgs &) {
     return gridder_rot_smem_bytes(NS, KBB) + size_t(NSM) * NS * NS * 4 + (NSM == 2 ? size_t(NS) * NS * 4 : 0);
 }
-template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int NSM = 0>
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int NSM = 0, int PKR = 0>
 cudaError_t launch_gridder_rot2(const KernelArgs &a, cudaStream_t st) {
-    return launch_tc(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, 1, NSM>, "gridder",
+    return launch_tc(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, 1, NSM, PKR>, "gridder",
                      smem_gridder_rot2<NS, WARPS, MT, MINB, KPT, GP, KBB, NSM>(a), WARPS * 32, a, st);
 }
 
@@ -1190,12 +1232,20 @@ cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
 #define TG(NS, W, MT, MB) \
     {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB>, 0, \
      smem_gridder_tc<NS, W, MT, MB>}
+#define TGROT2P(NS, W, MT, MB, KPT, GP, NSM, TAG) \
+    {NS, 8 * KPT, kTensor, 1, "gridder_rot2p<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP "," TAG ">", \
+     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM, 1>, 8 * KPT, smem_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM>}
 const Variant kTcGridder[] = {
     TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
     TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TG(24, 12, 3, 2), TG(32, 16, 4, 2), TG(16, 4, 4, 4),
+    // packed rotation (selected by name while measured)
+    TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2P(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2P(32, 16, 4, 2, 2, 2, 2, "lmnsm"),
+    TGROT2P(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2P(32, 32, 2, 1, 4, 2, 1, "nsm"), TGROT2P(32, 32, 2, 1, 4, 4, 0, "r"),
+    TGROT2P(24, 12, 3, 2, 4, 4, 0, "r"), TGROT2P(16, 8, 2, 2, 2, 2, 0, "r"),
 };
+#undef TGROT2P
 #undef TGROT2
 #undef TGROT2N
 #undef TG
