@@ -508,7 +508,9 @@ __device__ __forceinline__ f2p add2(f2p a, f2p b) {
 // pair of FFMA2 / FMUL2 (4 instead of 8 scalar instructions), and E^j D_j is accumulated as
 // acc += Re(E^j) D_j, acc2 += Im(E^j) D_j on the (re, im) pairs the mma writes (two FFMA2 with a
 // broadcast operand instead of four FFMA per pixel row); i acc2 joins acc once per item (complex
-// multiplication by i is linear).  The same products, half the instructions of the rotation.
+// multiplication by i is linear).  The same products, half the instructions of the rotation -- but the
+// extra accumulators spill at 64-80 registers: measured LOFAR 32.4 -> 36.6 ms, SKA-T1024 145 -> 157-192 ms
+// (sweep r02f), so PKR = 0 stays the default.
 template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB, int TU = 1, int NSM = 0,
           int PKR = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const KernelArgs a) {
@@ -1240,10 +1242,8 @@ const Variant kTcGridder[] = {
     TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TG(24, 12, 3, 2), TG(32, 16, 4, 2), TG(16, 4, 4, 4),
-    // packed rotation (selected by name while measured)
-    TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2P(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2P(32, 16, 4, 2, 2, 2, 2, "lmnsm"),
-    TGROT2P(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2P(32, 32, 2, 1, 4, 2, 1, "nsm"), TGROT2P(32, 32, 2, 1, 4, 4, 0, "r"),
-    TGROT2P(24, 12, 3, 2, 4, 4, 0, "r"), TGROT2P(16, 8, 2, 2, 2, 2, 0, "r"),
+    // packed rotation (measured slower: register spills outweigh the saved FFMA; selected by name only)
+    TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2P(32, 32, 2, 1, 4, 4, 0, "r"),
 };
 #undef TGROT2P
 #undef TGROT2
