@@ -443,6 +443,11 @@ def run_ours(args):
                  "paper_context": "P:258: gridder + degridder > 93% of the cycle on Haswell / Fiji / Pascal"}
         del tap_img
 
+    # ---- the host adder / splitter: grid in host memory ----------------------------------------
+    host_adder = None
+    if args.host_adder and kind == "grid+degrid" and world == 1:
+        host_adder = run_host_adder(args, idg, obs, plan, vis_d, uvw_d, at_d, tp_d, dev, nvis_rank)
+
     # ---- e2e: host buffers through the public API ------------------------------------------------
     bufs = {"vis": vis_d, "out": out_d}
     del vis_d, out_d
@@ -536,7 +541,7 @@ def run_ours(args):
         "grid_mvis_s": per_kernel.get("gridder", {}).get("mvis_s"),
         "degrid_mvis_s": per_kernel.get("degridder", {}).get("mvis_s"),
         "plan_s": plan_s, "clocks": clocks.summary(), "energy": energy, "e2e": e2e, "gpu_launches": gpu_launches,
-        "imaging_cycle": cycle,
+        "imaging_cycle": cycle, "host_adder": host_adder,
         "roofline": roofline, "kernels": per_kernel, "rho_sweep_TOps_s": rho_sweep or None,
         "cpu_baseline": cpu,
     }
@@ -544,6 +549,48 @@ def run_ours(args):
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def run_host_adder(args, idg, obs, plan, vis_d, uvw_d, at_d, tp_d, dev, nvis):
+    """grid + degrid with the grid in HOST memory (idg_grid_host_adder / idg_degrid_host_splitter):
+    visibilities from page-locked host memory, subgrids streamed to / from the host and added / split by
+    host threads.  Wall-clock per step (the host adds are part of the call), MVis/s."""
+    import torch
+    try:
+        import psutil
+        avail = psutil.virtual_memory().available
+    except Exception:
+        avail = None
+    vis_bytes = vis_d.numel() * 8
+    grid_bytes = 4 * obs.grid_size * obs.grid_size * 8
+    if avail is not None and 2 * vis_bytes + grid_bytes > 0.6 * avail:
+        return {"value": None, "skipped": "host memory"}
+    vis_h, r1 = host_buffer(tuple(vis_d.shape), torch.complex64)
+    out_h, r2 = host_buffer(tuple(vis_d.shape), torch.complex64)
+    vis_h.copy_(vis_d)
+    grid_h = torch.zeros((4, obs.grid_size, obs.grid_size), dtype=torch.complex64)
+    ws = idg.adder_workspace(plan, dev, buffers=8)
+    times = []
+    for k in range(1 + max(1, args.host_adder_steps)):
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        grid_h.zero_()
+        idg.grid_host_adder(plan, vis_h, uvw_d, at_d, tp_d, grid_h, ws)
+        idg.degrid_host_splitter(plan, grid_h, uvw_d, at_d, tp_d, out_h, ws)
+        torch.cuda.synchronize(dev)
+        if k > 0:
+            times.append(time.perf_counter() - t0)
+    res = {"value": nvis / statistics.median(times) / 1e6, "unit": "MVis/s", "steps": len(times),
+           "s_per_step": statistics.median(times), "host_threads": int(os.environ.get("IDG_HOST_THREADS", "0")) or
+           min(32, os.cpu_count() or 1),
+           "subgrid_bytes_per_step": int(2 * plan.nr_subgrids * 4 * obs.subgrid_size ** 2 * 8),
+           "api": "idg_grid_host_adder + idg_degrid_host_splitter (grid in host memory; wall clock per step)"}
+    for t, r in ((vis_h, r1), (out_h, r2)):
+        if r:
+            unregister_host(t)
+    del vis_h, out_h, grid_h, ws
+    torch.cuda.empty_cache()
+    return res
 
 
 def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, world, rank, nvis_total, bufs,
@@ -722,6 +769,9 @@ def main():
     ap.add_argument("--no-rho-sweep", action="store_true")
     ap.add_argument("--no-kernel-energy", action="store_true")
     ap.add_argument("--no-imaging-cycle", action="store_true")
+    ap.add_argument("--host-adder", action="store_true",
+                    help="also time grid + degrid with the grid in host memory (host adder / splitter, P:226)")
+    ap.add_argument("--host-adder-steps", type=int, default=3)
     ap.add_argument("--energy-launches", type=int, default=5)
     ap.add_argument("--timesteps", type=int, default=0,
                     help="tuning only: override the config's T (the line then names the reduced workload)")

@@ -1244,6 +1244,8 @@ const Variant kTcGridder[] = {
     TG(24, 12, 3, 2), TG(32, 16, 4, 2), TG(16, 4, 4, 4),
     // packed rotation (measured slower: register spills outweigh the saved FFMA; selected by name only)
     TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2P(32, 32, 2, 1, 4, 4, 0, "r"),
+    // group-pass experiments for N~ = 32 (selected by name only)
+    TGROT2N(32, 16, 4, 2, 4, 1, 1, "nsm"), TGROT2N(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2N(32, 32, 2, 1, 4, 2, 1, "nsm"),
 };
 #undef TGROT2P
 #undef TGROT2
@@ -1275,8 +1277,10 @@ const Variant kTcDegridder[] = {
     TDROTC(24, 8, 4, 1, 4, 4, "degridder_rot"), TDROTC(32, 16, 2, 1, 4, 4, "degridder_rot"),
     TDROTC(16, 8, 4, 1, 4, 4, "degridder_rot"),
     TD(24, 8, 2, 4), TD(32, 8, 4, 2), TD(16, 8, 4, 2),
-    // the single-chain N~ = 32 kernels (selected by name only)
+    // the single-chain N~ = 32 kernels, and 8-row units for 16-channel items (finer work units for short
+    // items) -- selected by name only
     TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"),
+    TDROTC(24, 8, 2, 1, 16, 8, "degridder_rot8"), TDROTC(24, 4, 3, 2, 16, 8, "degridder_rot8"),
 };
 #undef TDROTC
 #undef TDROTX
