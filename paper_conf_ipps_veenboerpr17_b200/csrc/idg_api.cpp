@@ -163,6 +163,7 @@ struct idg_plan {
     int64_t nr_vis_assigned = 0, nr_vis_dropped = 0, nr_pairs = 0;
     int32_t max_channels_in_item = 0;
     int32_t max_timesteps_in_item = 0;
+    float mean_timesteps_in_item = 0.0f;
     std::vector<int64_t> dropped;    // [nr][2]: (offset, count) in visibilities of every dropped run,
                                      // split at baseline boundaries (R-12, R-13: predicted as 0)
     std::vector<WorkGroup> groups;   // host-streamed work groups
@@ -393,6 +394,7 @@ idg::KernelArgs make_args(const idg_plan *plan, const DeviceCopy *dc, const floa
     a.grid = static_cast<float2 *>(d_grid);
     a.max_channels_in_item = plan->max_channels_in_item;
     a.max_timesteps_in_item = plan->max_timesteps_in_item;
+    a.mean_timesteps_in_item = plan->mean_timesteps_in_item;
     a.channel_gcd = plan->channel_gcd;
     a.channels_uniform = plan->channels_uniform;
     a.channel_step = plan->channel_step;
@@ -476,14 +478,17 @@ idg_status idg_plan_create(const idg_plan_params *params, int32_t nr_stations, i
         plan->nr_vis_dropped = res.nr_vis_dropped;
         const int64_t npix = int64_t(params->subgrid_size) * params->subgrid_size;
         int g = 0;
+        double sum_t = 0.0;
         for (const auto &it : plan->items) {
             const int nc = it.channel_end - it.channel_begin;
             plan->nr_pairs += npix * it.nr_timesteps * nc;
             plan->max_channels_in_item = std::max(plan->max_channels_in_item, nc);
             plan->max_timesteps_in_item = std::max(plan->max_timesteps_in_item, it.nr_timesteps);
+            sum_t += double(it.nr_timesteps);
             g = std::gcd(g, nc);
         }
         plan->channel_gcd = g == 0 ? 1 : g;
+        plan->mean_timesteps_in_item = plan->items.empty() ? 0.0f : float(sum_t / double(plan->items.size()));
         // uniform channel spacing (enables the phasor recurrence over channels in the gridder)
         // (every nu_c within 1e-12 nu_0 of nu_0 + c d: the kernels that rotate phasors across channels
         // then see phase errors below 2 pi |u| 1e-12 nu_0 C / c * L/2 ~ 1e-6 rad at the configs)

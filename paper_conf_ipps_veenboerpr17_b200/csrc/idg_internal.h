@@ -51,6 +51,7 @@ struct KernelArgs {
                                  // degridders read their split subgrids from here (host adder / splitter)
     int32_t max_channels_in_item;
     int32_t max_timesteps_in_item;
+    float mean_timesteps_in_item; // mean T~ over the items (short-item kernel choice)
     int32_t channel_gcd;         // gcd of all items' channel counts
     int32_t channels_uniform;    // 1 if nu_c = nu_0 + c d for all c (to 1e-12 nu_0)
     float channel_step;          // (nu_{c+1} - nu_c) / c  [1/m], valid when channels_uniform
@@ -68,6 +69,7 @@ struct Variant {
     Launcher fn;
     int max_channels = 0;  // > 0: every item has at most this many channels (unrolled channel groups)
     SmemFn smem = nullptr; // dynamic shared memory of a launch (the plan's items must fit the device)
+    int max_mean_timesteps = 0;  // > 0: eligible only when the items' mean T~ is at most this (short items)
 };
 // Tensor-core variants (idg_kernels_tc.cu); the first eligible one is the default.
 const Variant *tc_gridder_variants(int *n);     // split-f16 mma (idg_kernels_tc.cu)

@@ -336,6 +336,7 @@ bool eligible(const Variant &var, const KernelArgs &a) {
     if (var.needs_uniform && !a.channels_uniform) return false;
     if (var.max_channels > 0 && a.max_channels_in_item > var.max_channels) return false;
     if (var.v != 0 && a.channel_gcd % var.v != 0) return false;
+    if (var.max_mean_timesteps > 0 && a.mean_timesteps_in_item > float(var.max_mean_timesteps)) return false;
     // shared memory grows with the plan's largest item (T~ for the degridders, C~ for the gridders): a
     // variant whose launch would not fit is skipped, so a kernel that fits (ultimately SIMT) runs instead
     if (var.smem) {

@@ -511,8 +511,13 @@ __device__ __forceinline__ f2p add2(f2p a, f2p b) {
 // multiplication by i is linear).  The same products, half the instructions of the rotation -- but the
 // extra accumulators spill at 64-80 registers: measured LOFAR 32.4 -> 36.6 ms, SKA-T1024 145 -> 157-192 ms
 // (sweep r02f), so PKR = 0 stays the default.
+// HOR = 1: the rotated groups are summed in Horner form, sum_j E^j D_j = D_0 + E (D_1 + E (D_2 + E D_3)),
+// passes in descending group order: one complex multiply-add by E per group (4 FFMA per pixel row) instead
+// of advancing E^j (4 FMUL / FFMA) and multiplying by it (4 FFMA).  Same value in exact arithmetic; the
+// rounding of J - 1 complex products either way.  Measured (SKA, J = 4): 1162 -> 1125 ms per launch (r02j);
+// for J = 2 both forms are the same 4 FFMA per row.
 template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB, int TU = 1, int NSM = 0,
-          int PKR = 0>
+          int PKR = 0, int HOR = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const KernelArgs a) {
     constexpr int NT = WARPS * 32;
     constexpr int NPIX = NS * NS;
@@ -642,8 +647,9 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
 #pragma unroll
             for (int i = 0; i < MT; ++i) {
                 uint4 bf0[GP];   // B fragments of the first pass, loaded ahead of the sincos
+                constexpr int FIRST = HOR ? KPT - GP : 0;
 #pragma unroll
-                for (int j = 0; j < GP; ++j) bf0[j] = fr[j * 32];
+                for (int j = 0; j < GP; ++j) bf0[j] = fr[(FIRST + j) * 32];
                 f2p nv = pn[i], lv = pl[i], mv = pm[i];
                 if constexpr (NSM) {
                     // re-read every timestep (volatile: not hoisted into registers, which is the point)
@@ -666,6 +672,58 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const Ke
                 for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[j], al[j]);
                 if constexpr (KPT == 1) {
                     mma3(acc[i], ah, al, bf0[0]);
+                } else if constexpr (HOR) {
+                    float2 er = make_float2(1.0f, 1.0f), ei = make_float2(0.0f, 0.0f);   // E_t of rows (g, g+8)
+                    float h[4];   // Horner sum of the groups j >= 1: rows g (h0, h1) and g+8 (h2, h3)
+#pragma unroll
+                    for (int p0 = KPT - GP; p0 >= 0; p0 -= GP) {
+                        uint4 bf[GP];
+                        float d[GP][4];
+#pragma unroll
+                        for (int j = 0; j < GP; ++j) bf[j] = p0 == KPT - GP ? bf0[j] : fr[(p0 + j) * 32];
+#pragma unroll
+                        for (int k = 0; k < 3; ++k) {
+                            const uint32_t *A = k < 2 ? ah : al;
+#pragma unroll
+                            for (int j = 0; j < GP; ++j) {
+                                const uint32_t b0 = k == 1 ? bf[j].z : bf[j].x, b1 = k == 1 ? bf[j].w : bf[j].y;
+                                if (p0 + j == 0)
+                                    mma16816(acc[i], A[0], A[1], A[2], A[3], b0, b1);
+                                else if (k == 0)
+                                    mma16816_zero(d[j], A[0], A[1], A[2], A[3], b0, b1);
+                                else
+                                    mma16816(d[j], A[0], A[1], A[2], A[3], b0, b1);
+                            }
+                        }
+                        if (p0 == KPT - GP) {
+                            // E4 = Phi(q+4) conj(Phi(q)), E = E4^2, packed over rows (g, g+8)
+                            const f2p C0 = pk(cs[0], cs[1]), S0 = pk(sn[0], sn[1]);
+                            const f2p C4 = pk(cs[2], cs[3]), S4 = pk(sn[2], sn[3]);
+                            const f2p r4 = fma2(C4, C0, mul2(S4, S0));
+                            const f2p i4 = sub2(mul2(S4, C0), mul2(C4, S0));
+                            er = unpk(sub2(mul2(r4, r4), mul2(i4, i4)));
+                            ei = unpk(mul2(add2(r4, r4), i4));
+                        }
+#pragma unroll
+                        for (int j = GP - 1; j >= 0; --j) {
+                            if (p0 + j == 0) continue;
+                            if (p0 + j == KPT - 1) {
+#pragma unroll
+                                for (int k = 0; k < 4; ++k) h[k] = d[j][k];
+                            } else {   // h = D_j + E h
+                                const float h0 = fmaf(er.x, h[0], fmaf(-ei.x, h[1], d[j][0]));
+                                const float h1 = fmaf(er.x, h[1], fmaf(ei.x, h[0], d[j][1]));
+                                const float h2 = fmaf(er.y, h[2], fmaf(-ei.y, h[3], d[j][2]));
+                                const float h3 = fmaf(er.y, h[3], fmaf(ei.y, h[2], d[j][3]));
+                                h[0] = h0; h[1] = h1; h[2] = h2; h[3] = h3;
+                            }
+                        }
+                    }
+                    // acc += E h (group 0 was accumulated in place by its mma)
+                    acc[i][0] = fmaf(er.x, h[0], fmaf(-ei.x, h[1], acc[i][0]));
+                    acc[i][1] = fmaf(er.x, h[1], fmaf(ei.x, h[0], acc[i][1]));
+                    acc[i][2] = fmaf(er.y, h[2], fmaf(-ei.y, h[3], acc[i][2]));
+                    acc[i][3] = fmaf(er.y, h[3], fmaf(ei.y, h[2], acc[i][3]));
                 } else {
                     float2 er, ei;   // E_t of rows (g, g+8)
                     float pr0 = 1.0f, pi0 = 0.0f, pr1 = 1.0f, pi1 = 0.0f;   // E^j of rows g, g+8
@@ -1202,9 +1260,10 @@ template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBat
 size_t smem_gridder_rot2(const KernelArgs &) {
     return gridder_rot_smem_bytes(NS, KBB) + size_t(NSM) * NS * NS * 4 + (NSM == 2 ? size_t(NS) * NS * 4 : 0);
 }
-template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int NSM = 0, int PKR = 0>
+template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB = kTcBatchKB, int NSM = 0, int PKR = 0,
+          int HOR = 0>
 cudaError_t launch_gridder_rot2(const KernelArgs &a, cudaStream_t st) {
-    return launch_tc(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, 1, NSM, PKR>, "gridder",
+    return launch_tc(gridder_rot2_kernel<NS, WARPS, MT, MINB, KPT, GP, KBB, 1, NSM, PKR, HOR>, "gridder",
                      smem_gridder_rot2<NS, WARPS, MT, MINB, KPT, GP, KBB, NSM>(a), WARPS * 32, a, st);
 }
 
@@ -1234,19 +1293,25 @@ cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
 #define TG(NS, W, MT, MB) \
     {NS, 8, kTensor, 0, "gridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_gridder_tc<NS, W, MT, MB>, 0, \
      smem_gridder_tc<NS, W, MT, MB>}
+#define TGROT2H(NS, W, MT, MB, KPT, GP, NSM, TAG) \
+    {NS, 8 * KPT, kTensor, 1, "gridder_rot2h<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP "," TAG ">", \
+     launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM, 0, 1>, 8 * KPT, smem_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM>}
 #define TGROT2P(NS, W, MT, MB, KPT, GP, NSM, TAG) \
     {NS, 8 * KPT, kTensor, 1, "gridder_rot2p<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ",GP" #GP "," TAG ">", \
      launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM, 1>, 8 * KPT, smem_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM>}
 const Variant kTcGridder[] = {
     TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
-    TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
+    TGROT2H(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TG(24, 12, 3, 2), TG(32, 16, 4, 2), TG(16, 4, 4, 4),
     // packed rotation (measured slower: register spills outweigh the saved FFMA; selected by name only)
     TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2P(32, 32, 2, 1, 4, 4, 0, "r"),
     // group-pass experiments for N~ = 32 (selected by name only)
     TGROT2N(32, 16, 4, 2, 4, 1, 1, "nsm"), TGROT2N(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2N(32, 32, 2, 1, 4, 2, 1, "nsm"),
+    // the E^j form for N~ = 32 (the default before the Horner form; selected by name only)
+    TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"),
 };
+#undef TGROT2H
 #undef TGROT2P
 #undef TGROT2
 #undef TGROT2N
@@ -1258,6 +1323,11 @@ const Variant kTcGridder[] = {
 #define TDROTC(NS, W, MB, U, CPT, R, TAG) \
     {NS, CPT, kTensor, 1, TAG "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, R>, CPT, smem_degridder_tc<NS>}
+// short items (the plan's mean T~ <= 64): 8 channel rows per lane, 4-timestep warp units (finer than the 8 of
+// R = 16, so ragged item tails leave fewer warps idle): lofar_short 3081 -> 3203 MVis/s, LOFAR -7% (r02i)
+#define TDROTS(NS, W, MB, U, CPT, R) \
+    {NS, CPT, kTensor, 1, "degridder_rot8<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, R>, CPT, smem_degridder_tc<NS>, 64}
 #define TDROTX(NS, W, MB, U, CPT, R, SCH) \
     {NS, CPT, kTensor, 1, "degridder_rot16s" #SCH "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, R, SCH>, CPT, smem_degridder_tc<NS>}
@@ -1268,7 +1338,7 @@ const Variant kTcGridder[] = {
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>, 0, \
      smem_degridder_tc<NS>}
 const Variant kTcDegridder[] = {
-    TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 1, 32, 16, 2),
+    TDROTS(24, 4, 3, 2, 16, 8), TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 1, 32, 16, 2),
     TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
     TDROTC(24, 8, 2, 1, 8, 8, "degridder_rot8"), TDROTC(32, 16, 2, 1, 8, 8, "degridder_rot8"),
@@ -1280,9 +1350,10 @@ const Variant kTcDegridder[] = {
     // the single-chain N~ = 32 kernels, and 8-row units for 16-channel items (finer work units for short
     // items) -- selected by name only
     TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"),
-    TDROTC(24, 8, 2, 1, 16, 8, "degridder_rot8"), TDROTC(24, 4, 3, 2, 16, 8, "degridder_rot8"),
+    TDROTC(24, 8, 2, 1, 16, 8, "degridder_rot8"),
 };
 #undef TDROTC
+#undef TDROTS
 #undef TDROTX
 #undef TDROT
 #undef TD
