@@ -1308,8 +1308,10 @@ const Variant kTcGridder[] = {
     TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2P(32, 32, 2, 1, 4, 4, 0, "r"),
     // group-pass experiments for N~ = 32 (selected by name only)
     TGROT2N(32, 16, 4, 2, 4, 1, 1, "nsm"), TGROT2N(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2N(32, 32, 2, 1, 4, 2, 1, "nsm"),
-    // the E^j form for N~ = 32 (the default before the Horner form; selected by name only)
-    TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"),
+    // the E^j form for N~ = 32 (the default before the Horner form), Horner with l, m, n from shared memory,
+    // Horner for predict's 16-channel items (selected by name only)
+    TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 4, 2, "lmnsm"), TGROT2H(32, 16, 4, 2, 4, 2, 0, "r"),
+    TGROT2H(32, 16, 4, 2, 2, 2, 2, "lmnsm"),
 };
 #undef TGROT2H
 #undef TGROT2P
