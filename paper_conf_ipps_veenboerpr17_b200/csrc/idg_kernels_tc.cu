@@ -514,8 +514,9 @@ __device__ __forceinline__ f2p add2(f2p a, f2p b) {
 // HOR = 1: the rotated groups are summed in Horner form, sum_j E^j D_j = D_0 + E (D_1 + E (D_2 + E D_3)),
 // passes in descending group order: one complex multiply-add by E per group (4 FFMA per pixel row) instead
 // of advancing E^j (4 FMUL / FFMA) and multiplying by it (4 FFMA).  Same value in exact arithmetic; the
-// rounding of J - 1 complex products either way.  Measured (SKA, J = 4): 1162 -> 1125 ms per launch (r02j);
-// for J = 2 both forms are the same 4 FFMA per row.
+// rounding of J - 1 complex products either way.  Measured (SKA, J = 4): 1162 -> 1125 ms per launch (r02j),
+// SKA-T1024 145.2 -> 139.7 ms (nsm) -> 135.6 ms (lmnsm: fewer spills, r02l); for J = 2 both forms are the
+// same 4 FFMA per row (predict: equal).
 template <int NS, int WARPS, int MT, int MINB, int KPT, int GP, int KBB_ = kTcBatchKB, int TU = 1, int NSM = 0,
           int PKR = 0, int HOR = 0>
 __global__ void __launch_bounds__(WARPS * 32, MINB) gridder_rot2_kernel(const KernelArgs a) {
@@ -1301,7 +1302,7 @@ cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
      launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM, 1>, 8 * KPT, smem_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM>}
 const Variant kTcGridder[] = {
     TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
-    TGROT2H(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
+    TGROT2H(32, 16, 4, 2, 4, 4, 2, "lmnsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TG(24, 12, 3, 2), TG(32, 16, 4, 2), TG(16, 4, 4, 4),
     // packed rotation (measured slower: register spills outweigh the saved FFMA; selected by name only)
@@ -1310,8 +1311,7 @@ const Variant kTcGridder[] = {
     TGROT2N(32, 16, 4, 2, 4, 1, 1, "nsm"), TGROT2N(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2N(32, 32, 2, 1, 4, 2, 1, "nsm"),
     // the E^j form for N~ = 32 (the default before the Horner form), Horner with l, m, n from shared memory,
     // Horner for predict's 16-channel items (selected by name only)
-    TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 4, 2, "lmnsm"), TGROT2H(32, 16, 4, 2, 4, 2, 0, "r"),
-    TGROT2H(32, 16, 4, 2, 2, 2, 2, "lmnsm"),
+    TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 2, 0, "r"),
 };
 #undef TGROT2H
 #undef TGROT2P
