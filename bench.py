@@ -764,7 +764,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-baseline-s", type=float, default=15.0)
-    ap.add_argument("--reference-step-s", type=float, default=8.0)
+    ap.add_argument("--reference-step-s", type=float, default=5.0)
     ap.add_argument("--rho-iterations", type=int, default=16384)
     ap.add_argument("--no-rho-sweep", action="store_true")
     ap.add_argument("--no-kernel-energy", action="store_true")
