@@ -619,13 +619,20 @@ def run_e2e(args, idg, parallel, obs, plan, kind, aterms, taper, dev, stream, wo
     # the same host arrays), else 2 rotating chunk buffers per direction
     need_full = local_world * (n_in + 1) * vis_bytes
     need_rot = local_world * (n_in + 1) * 2 * chunk_bytes
+    # 0: full host arrays, 1: rotating chunk buffers, 2: skip -- agreed over the ranks (the most conservative
+    # choice), since the collectives below must be entered by every rank alike
+    mode = 0
     if host_avail is not None and need_full > 0.7 * host_avail:
-        if nchunks == 1 or need_rot > 0.7 * host_avail:
-            return {"value": None, "unit": "MVis/s", "skipped": f"page-locked host buffers ({need_full / 1e9:.0f} GB for "
-                    f"{local_world} local ranks) do not fit the host ({host_avail / 1e9:.0f} GB available)"}
-        rotating = True
-    else:
-        rotating = False
+        mode = 2 if (nchunks == 1 or need_rot > 0.7 * host_avail) else 1
+    if world > 1:
+        tm = torch.tensor([mode], dtype=torch.int64, device=dev)
+        dist.all_reduce(tm, op=dist.ReduceOp.MAX)
+        mode = int(tm.item())
+    if mode == 2:
+        return {"value": None, "unit": "MVis/s", "skipped": f"page-locked host buffers ({need_full / 1e9:.0f} GB for "
+                f"{local_world} local ranks) do not fit the host "
+                f"({(host_avail or 0) / 1e9:.0f} GB available on this rank)"}
+    rotating = mode == 1
     t_plan = time.perf_counter()
     if nchunks == 1:
         cobs, cplans = [obs], [plan]
