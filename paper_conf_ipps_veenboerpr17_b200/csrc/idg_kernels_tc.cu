@@ -1305,13 +1305,11 @@ const Variant kTcGridder[] = {
     TGROT2H(32, 16, 4, 2, 4, 4, 2, "lmnsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TG(24, 12, 3, 2), TG(32, 16, 4, 2), TG(16, 4, 4, 4),
-    // packed rotation (measured slower: register spills outweigh the saved FFMA; selected by name only)
-    TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2P(32, 32, 2, 1, 4, 4, 0, "r"),
-    // group-pass experiments for N~ = 32 (selected by name only)
-    TGROT2N(32, 16, 4, 2, 4, 1, 1, "nsm"), TGROT2N(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2N(32, 32, 2, 1, 4, 2, 1, "nsm"),
-    // the E^j form for N~ = 32 (the default before the Horner form), Horner with l, m, n from shared memory,
-    // Horner for predict's 16-channel items (selected by name only)
-    TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 4, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 2, 0, "r"),
+    // alternates kept for measurement (selected by name only): the packed rotation (slower: spills), the
+    // E^j form for N~ = 32 (the default before the Horner form), Horner with n only in shared memory.
+    // Measured and dropped (r02i / r02o, SKA-T1024, against 135.7 ms): group passes of 1 / 4 in the E^j
+    // form, Horner at 16 warps / SM with 128 registers (138.0), 32 warps of 2 tiles (147.4).
+    TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 4, 1, "nsm"),
 };
 #undef TGROT2H
 #undef TGROT2P
