@@ -495,9 +495,16 @@ def run_ours(args):
         k["frac_sincos_fma_roofline"] = k["TOps_s"] / peak
     roofline = None
     if dominant:
+        traffic = (hw or {}).get("dram_bytes")
+        if traffic and (hw or {}).get("capture_timesteps"):
+            # the capture ran the same kernels at a shorter T: DRAM bytes scale with the visibilities
+            traffic = traffic * obs.nr_timesteps / hw["capture_timesteps"]
         roofline = {"bound": "alu", "kernel": dominant, "achieved": per_kernel[dominant]["TOps_s"],
                     "peak": peak, "unit": "TOps/s", "frac": per_kernel[dominant]["TOps_s"] / peak,
-                    "traffic": (hw or {}).get("dram_bytes"),
+                    "traffic": traffic,
+                    "traffic_source": "dram__bytes_read.sum + dram__bytes_write.sum of the dominant kernel, one ncu "
+                                      "--set full capture (profiles/ncu_summary.json), scaled to this T when the "
+                                      "capture ran a shorter T",
                     "peak_source": "the paper's sincos+FMA roofline (P:276-290) from B200 unit counts at the timed "
                                    "region's SM clock: 148 SMs x min(128 FMA lanes / 17, 16 MUFU lanes / 2) pairs/clk "
                                    "x 36 paper-ops per pair (P:258); a ceiling for the paper's formulation (17 FMA + "

@@ -144,6 +144,8 @@ def main():
     ap.add_argument("--config", default="lofar")
     ap.add_argument("--launches")
     ap.add_argument("--note", default="")
+    ap.add_argument("--capture-timesteps", type=int, default=0,
+                    help="T of the captured workload (bench.py scales dram_bytes to its own T)")
     ap.add_argument("--bench", help="bench.py JSON line of the same build: adds its CUDA-event shares")
     args = ap.parse_args()
     md = [f"# ncu summary {args.tag} ({args.config})", ""]
@@ -161,6 +163,8 @@ def main():
             short = "degridder" if "degridder" in rec["kernel"] else "gridder" if "gridder" in rec["kernel"] \
                 else rec["kernel"].split("(")[0]
             ent = {"tag": args.tag, "kernel": rec["kernel"], "dram_bytes": rec["dram_bytes"]}
+            if args.capture_timesteps:
+                ent["capture_timesteps"] = args.capture_timesteps
             if "_pipes" in rec:
                 p = rec["_pipes"]
                 bk = max(p, key=p.get)

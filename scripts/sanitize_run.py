@@ -24,6 +24,11 @@ def main():
         name, kw = "ska", dict(T=128, nr_stations=3)
     if name == "lofar_small":
         name, kw = "lofar", dict(T=256, nr_stations=4)
+    if name == "small_dde8":          # 8 channels: the N~ = 16 rotation gridder (KPT 1) and 8-row degridder
+        name, kw = "small_dde", dict(C=8)
+    select = None
+    if name == "short_items":         # long baselines of lofar_short: the short-item (mean T~ <= 64) degridder
+        name, select = "lofar_short", (3, 256, 2048)
     g, d = FAMILIES[fam]
     if g:
         os.environ["IDG_GRIDDER_VARIANT"], os.environ["IDG_DEGRIDDER_VARIANT"] = g, d
@@ -31,6 +36,8 @@ def main():
     import torch
     import paper_conf_ipps_veenboerpr17_b200 as idg
     obs = idgsynth.make_observation(name, **kw)
+    if select:
+        obs = obs.select(obs.longest_baselines(select[0]), nr_timesteps=select[1], time_begin=select[2])
     vis = idgsynth.make_visibilities(obs)
     aterms = idgsynth.make_aterms(obs, "random")
     taper = idgsynth.make_taper(obs.subgrid_size, "asymmetric")
