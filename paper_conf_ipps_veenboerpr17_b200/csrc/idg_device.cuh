@@ -88,15 +88,18 @@ __device__ __forceinline__ ItemSetup item_setup(const KernelArgs &a, int item, i
 }
 
 // B_t and Q_t coefficients (2 pi x wavelengths) of one timestep, formed in fp64.
-__device__ __forceinline__ void timestep_coefficients(const KernelArgs &a, const ItemSetup &s,
-                                                      int t, float4 &cB, float4 &cQ) {
-    const float *p = a.uvw + (int64_t(s.md.baseline) * a.nr_timesteps + t) * 3;
-    const float u = p[0], v = p[1], w = p[2];
+__device__ __forceinline__ void timestep_coefficients_uvw(const ItemSetup &s, float u, float v, float w,
+                                                          float4 &cB, float4 &cQ) {
     cB = make_float4(float(kTwoPi * (double(u) * s.f_ref - s.u0)),
                      float(kTwoPi * (double(v) * s.f_ref - s.v0)),
                      float(kTwoPi * (double(w) * s.f_ref - s.w0)), 0.0f);
     cQ = make_float4(float(kTwoPi * double(u)), float(kTwoPi * double(v)),
                      float(kTwoPi * double(w)), 0.0f);
+}
+__device__ __forceinline__ void timestep_coefficients(const KernelArgs &a, const ItemSetup &s,
+                                                      int t, float4 &cB, float4 &cQ) {
+    const float *p = a.uvw + (int64_t(s.md.baseline) * a.nr_timesteps + t) * 3;
+    timestep_coefficients_uvw(s, p[0], p[1], p[2], cB, cQ);
 }
 
 

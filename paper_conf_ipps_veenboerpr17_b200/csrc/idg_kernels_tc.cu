@@ -169,11 +169,12 @@ __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wai
 // One pass: in[r][x] = src[pol * N~^2 + a * RS + x * KS] for r = pol N~ + a, multiplied by `scale`
 // (power of two: f16 range); emit(pol, a, k, out[r][k] * outmul) for every output.  Warps take 16x8
 // output tiles round robin.
-template <int NS, int WARPS, typename Emit>
+// NP < 4: the first NP polarisations of src only (rows r = pol N~ + a, pol < NP).
+template <int NS, int WARPS, int NP = 4, typename Emit>
 __device__ __forceinline__ void dft_pass_tc(const float2 *src, int RS, int KS, const uint4 *tab, float scale,
                                             float outmul, Emit emit) {
     constexpr int NPIX = NS * NS;
-    constexpr int MTL = NS / 4, NTL = NS / 4, KST = NS / 8;
+    constexpr int MTL = NP * NS / 16, NTL = NS / 4, KST = NS / 8;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
     for (int tile = warp; tile < MTL * NTL; tile += WARPS) {
         const int mt = tile / NTL, nt = tile - mt * NTL;
@@ -1285,6 +1286,11 @@ cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
 // Gridders.  First eligible entry is the default: the rotation gridder when every item has exactly 8 KPT
 // uniformly spaced channels (nsm / lmnsm: pixel coordinates re-read from shared memory, N~ = 32), else
 // the direct kernel (one sincos per pair; any channel table with C~ % 8 == 0), else the SIMT kernel.
+#include "idg_kernels_umma.cuh"   // the tcgen05 rotation gridder (gridder_umma_rot), in this namespace
+
+#define GUR(KPT) \
+    {32, 8 * KPT, kTensor, 1, "gridder_umma_rot<32,KPT" #KPT ",pair>", launch_gridder_umma_rot<KPT>, 8 * KPT, \
+     smem_gridder_umma_rot<KPT>}
 #define TGROT2(NS, W, MT, MB, KPT) \
     {NS, 8 * KPT, kTensor, 1, "gridder_rot2<" #NS ",W" #W ",MT" #MT ",minB" #MB ",KPT" #KPT ">", \
      launch_gridder_rot2<NS, W, MT, MB, KPT, KPT, 128>, 8 * KPT, smem_gridder_rot2<NS, W, MT, MB, KPT, KPT, 128>}
@@ -1310,7 +1316,10 @@ const Variant kTcGridder[] = {
     // Measured and dropped (r02i / r02o, SKA-T1024, against 135.7 ms): group passes of 1 / 4 in the E^j
     // form, Horner at 16 warps / SM with 128 registers (138.0), 32 warps of 2 tiles (147.4).
     TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 4, 1, "nsm"),
+    // tcgen05 / TMEM rotation gridder (selected by name while measured)
+    GUR(4), GUR(2),
 };
+#undef GUR
 #undef TGROT2H
 #undef TGROT2P
 #undef TGROT2

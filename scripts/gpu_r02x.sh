@@ -1,0 +1,12 @@
+#!/bin/bash
+# Round-2 pass x: the final cluster-pair tcgen05 gridder (parity + SKA / predict timing against the defaults).
+set -u
+TAG=${1:-r02x}
+OUT=gpurun_out; mkdir -p $OUT
+python __graft_entry__.py > $OUT/build_$TAG.log 2>&1 || { echo BUILD FAILED; tail -20 $OUT/build_$TAG.log; exit 1; }
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -s -k "umma" -x > $OUT/pytest_umma_$TAG.log 2>&1; echo "pytest umma rc=$?"
+grep -E "grid\[umma\]|passed|failed|Error|error" $OUT/pytest_umma_$TAG.log | tail -8
+timeout 600 python scripts/variant_sweep.py --config ska --timesteps 1024 --which gridder --variants \
+  'gridder_rot2h<32,W16,MT4,minB2,KPT4,GP4,lmnsm>' 'gridder_umma_rot<32,KPT4,pair>' 2>&1 | tee $OUT/sweep_umma_$TAG.txt
+timeout 600 python scripts/variant_sweep.py --config predict --timesteps 256 --which gridder --variants \
+  'gridder_rot2<32,W16,MT4,minB2,KPT2,GP2,lmnsm>' 'gridder_umma_rot<32,KPT2,pair>' 2>&1 | tee -a $OUT/sweep_umma_$TAG.txt

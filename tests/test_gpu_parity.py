@@ -79,6 +79,7 @@ KINDS = {
     "default": (None, None),   # default: rotation kernels where the channel layout allows, else direct
     "tc": ("tc", "tc"),        # direct tensor-core kernels (one sincos per pair, any channel table)
     "simt": ("simt", "simt"),  # CUDA-core kernels (the paper's structure)
+    "umma": ("gridder_umma_rot<*", ""),  # tcgen05 / TMEM rotation gridder, cluster pair (N~ = 32, 16 / 32 ch)
 }
 
 
