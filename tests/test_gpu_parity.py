@@ -258,6 +258,26 @@ def test_host_adder_and_splitter(name, kw, chunk, drop, monkeypatch):
     assert torch.equal(v_host, v_dev.cpu())
 
 
+@pytest.mark.parametrize("name,kw", [("ska", dict(T=256, nr_stations=4)), ("predict", dict(T=128, nr_stations=4))])
+def test_host_adder_tcgen05_gridder(name, kw, monkeypatch):
+    """The cluster-pair tcgen05 gridder writes its two polarisation halves into the host adder's subgrid
+    buffer (slot = the item's position in the order, not the CTA index)."""
+    monkeypatch.setenv("IDG_HOST_CHUNK_BYTES", "2000000")
+    monkeypatch.setenv("IDG_GRIDDER_VARIANT", "gridder_umma_rot<*")
+    obs = idgsynth.make_observation(name, **kw)
+    vis, aterms, tap = _inputs(obs, "random", "asymmetric")
+    items, _ = oracle.plan(obs)
+    plan = idg.Plan.from_observation(obs)
+    ws = idg.adder_workspace(plan, buffers=3)
+    g_host = torch.zeros(oracle.grid_shape(obs), dtype=torch.complex64)
+    idg.grid_host_adder(plan, torch.from_numpy(vis).pin_memory(), _dev(obs.uvw), _dev(aterms), _dev(tap),
+                        g_host, ws)
+    assert idg.last_variant("gridder").startswith("gridder_umma_rot<")
+    err = rel_rms(g_host.numpy(), oracle.grid(obs, items, vis, aterms, tap))
+    print(f"host adder [umma] {name} {kw}: rel rms {err:.3e}")
+    assert err <= TOL, err
+
+
 def test_host_streamed_upload_waits_for_the_callers_stream():
     """A non-blocking device->host copy into vis_h queued on the caller's stream right before
     idg_grid_host (no synchronize in between): the uploads must see the new host data."""
