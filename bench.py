@@ -338,7 +338,22 @@ def run_ours(args):
         grid_d = idgsynth.torch_grid(obs, dev) if rank == 0 else torch.zeros((4, N, N), dtype=torch.complex64,
                                                                              device=dev)
 
+    # --exchange peer (N > 1): the banded grid -- every rank's gridder adds into the owners' row bands through
+    # CUDA-IPC peer memory and every degridder reads them, so no reduce / broadcast runs (parallel.BandedGrid)
+    banded = parallel.BandedGrid(plan, dev) if (world > 1 and args.exchange == "peer") else None
+    if banded is not None and kind != "grid+degrid":
+        banded.load(grid_d if rank == 0 else idgsynth.torch_grid(obs, dev))   # every rank its band of the model
+
     def step():
+        if banded is not None:
+            if kind == "grid+degrid":
+                banded.sync()                                            # no peer still reads the bands
+                banded.band.zero_()
+                banded.sync()                                            # every band zeroed before any add
+                banded.grid(vis_d, uvw_d, at_d, tp_d)                    # adder into the owners' bands
+                banded.sync()                                            # every rank's adds have landed
+            banded.degrid(uvw_d, at_d, tp_d, out_d)                      # splitter reads the owners' bands
+            return
         if kind == "grid+degrid":
             grid_d.zero_()
             sharded.grid(vis_d, uvw_d, at_d, tp_d, grid_d, dst=0)        # + NCCL reduce of the uv-grids
@@ -370,6 +385,9 @@ def run_ours(args):
     idg.profiling_enable(False)
     gpu_launches = idg.launch_count() - launches0
     kern = idg.profiling_read()
+    if banded is not None:
+        banded.sync()                 # no rank still reads a peer's band
+        banded.close()
     ms = ev0.elapsed_time(ev1)
     t = torch.tensor([ms], dtype=torch.float64, device=dev)
     if world > 1:
@@ -542,7 +560,9 @@ def run_ours(args):
                                        "median": float(np.median(md["nr_timesteps"])) if len(md) else 0.0,
                                        "hist_bins_of_16": (np.bincount(np.minimum(md["nr_timesteps"], 128) // 16,
                                                                        minlength=9) / max(1, len(md))).round(4).tolist()},
-                   "parallelism": f"baseline shards x{world}" + (" + NCCL reduce/broadcast" if world > 1 else ""),
+                   "parallelism": f"baseline shards x{world}" + (
+                       "" if world == 1 else " + banded grid, adder / splitter into the owners' bands over peer "
+                       "memory (no collective; e2e: NCCL)" if banded is not None else " + NCCL reduce/broadcast"),
                    "l2": f"inputs larger than L2 (visibilities {vis_bytes / 1e9:.1f} GB/step)",
                    "degrid_in_place": inplace},
         "grid_mvis_s": per_kernel.get("gridder", {}).get("mvis_s"),
@@ -783,6 +803,9 @@ def main():
     ap.add_argument("--no-rho-sweep", action="store_true")
     ap.add_argument("--no-kernel-energy", action="store_true")
     ap.add_argument("--no-imaging-cycle", action="store_true")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "peer"],
+                    help="N > 1: NCCL reduce / broadcast of the covered grid band (default), or the banded grid "
+                         "with the exchange fused into the kernels (peer memory)")
     ap.add_argument("--host-adder", action="store_true",
                     help="also time grid + degrid with the grid in host memory (host adder / splitter, P:226)")
     ap.add_argument("--host-adder-steps", type=int, default=3)

@@ -140,6 +140,42 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
                       size_t workspace_bytes, idg_stream stream);
 
 /*
+ * Banded grid: the multi-GPU exchange fused into the kernels.  The work is split over devices by
+ * baselines ("embarrassingly parallel"); what couples the devices is the adder, which sums
+ * every subgrid into the one uv-grid, and, for prediction, every device reading the one model grid.
+ * Here the grid is distributed by row bands: band r holds grid rows [r R, (r+1) R) of every [plane][pol]
+ * as complex64 [nz][4][R][N] (R = band_rows), and the adder of every work item adds each subgrid row
+ * straight into the band that owns it -- another rank's memory when d_bands holds CUDA-IPC mappings
+ * (idg_ipc_open; NVLink / NVSwitch peer access) -- so the cross-rank reduction happens inside the gridder;
+ * the degridder's splitter reads the owners' bands the same way (no broadcast).
+ *   d_bands    DEVICE array of nr_bands device pointers (nr_bands * band_rows >= N); the pointers may be
+ *              peer mappings; the caller keeps them valid for the call
+ *   idg_grid_bands    the bands are ACCUMULATED (scalar fp32 atomics, order unspecified: R-19); they are
+ *                     complete for readers once every rank's call has completed (synchronise, then a
+ *                     cross-rank barrier)
+ *   idg_degrid_bands  the bands are read only; d_vis OVERWRITTEN as idg_degrid
+ * Other arguments as idg_grid / idg_degrid.  Errors: IDG_ERR_INVALID_ARG for NULL pointers or bands that
+ * do not cover the grid; IDG_ERR_CUDA for launch failures (asynchronous faults surface at the next sync).
+ */
+idg_status idg_grid_bands(const idg_plan *plan, const void *d_vis, const float *d_uvw, const void *d_aterms,
+                          const float *d_taper, void *const *d_bands, int32_t nr_bands, int32_t band_rows,
+                          idg_stream stream);
+idg_status idg_degrid_bands(const idg_plan *plan, const void *const *d_bands, int32_t nr_bands,
+                            int32_t band_rows, const float *d_uvw, const void *d_aterms, const float *d_taper,
+                            void *d_vis, idg_stream stream);
+
+/*
+ * CUDA IPC for the bands.  idg_ipc_handle: the 64-byte cudaIpcMemHandle_t of the allocation containing
+ * d_ptr and d_ptr's byte offset in it (handles name whole allocations, e.g. a caching allocator's
+ * segment).  idg_ipc_open: map another process's allocation (peer access enabled lazily) and return the
+ * pointer at `offset`; not for the calling process's own allocations.  idg_ipc_close: unmap (same offset).
+ * Errors: IDG_ERR_INVALID_ARG for NULL arguments, IDG_ERR_CUDA when the runtime refuses.
+ */
+idg_status idg_ipc_handle(const void *d_ptr, unsigned char handle[64], uint64_t *offset);
+idg_status idg_ipc_open(const unsigned char handle[64], uint64_t offset, void **d_ptr);
+idg_status idg_ipc_close(void *d_ptr, uint64_t offset);
+
+/*
  * Host-streamed calls: the paper's asynchronous I/O (Fig. 7).  The visibilities live in
  * HOST memory (page-locked for overlap, e.g. cudaHostAlloc / torch pin_memory) and stream through
  * triple-buffered device staging buffers in work groups of contiguous baselines: uploads on an

@@ -628,6 +628,124 @@ idg_status idg_degrid(const idg_plan *plan, const void *d_grid, const float *d_u
 }
 
 // ------------------------------------------------------------------------------------------------
+// Banded grid (peer memory): the grid is distributed over the ranks by row bands and the adder / splitter
+// of every work item goes straight to the owner's band -- the cross-rank sum of the gridded subgrids
+// (the adder, independent work split over devices) and the model-grid broadcast of the
+// degridding step are fused into the kernels instead of following them as collectives.
+// ------------------------------------------------------------------------------------------------
+static idg_status validate_bands(const idg_plan *plan, const void *bands, int32_t nr_bands, int32_t band_rows) {
+    if (!bands) return fail(IDG_ERR_INVALID_ARG, "d_bands is NULL");
+    if (nr_bands < 1 || band_rows < 1)
+        return fail(IDG_ERR_INVALID_ARG, "nr_bands and band_rows must be >= 1");
+    if (int64_t(nr_bands) * band_rows < plan->params.grid_size)
+        return fail(IDG_ERR_INVALID_ARG, "nr_bands * band_rows must cover the grid_size rows");
+    return IDG_OK;
+}
+
+idg_status idg_grid_bands(const idg_plan *plan, const void *d_vis, const float *d_uvw, const void *d_aterms,
+                          const float *d_taper, void *const *d_bands, int32_t nr_bands, int32_t band_rows,
+                          idg_stream stream) {
+    try {
+        idg_status st = validate_call(plan, d_vis, d_uvw, d_aterms, d_taper, d_bands);
+        if (st != IDG_OK) return st;
+        if ((st = validate_bands(plan, d_bands, nr_bands, band_rows)) != IDG_OK || plan->items.empty()) return st;
+        const DeviceCopy *dc = nullptr;
+        if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper, const_cast<void *>(d_vis), nullptr);
+        a.bands = reinterpret_cast<float2 *const *>(d_bands);
+        a.band_rows = band_rows;
+        cudaError_t e = idg::launch_gridder(a, reinterpret_cast<cudaStream_t>(stream));
+        if (e != cudaSuccess) return cuda_fail(e, "gridder launch (banded)");
+        return IDG_OK;
+    } catch (const std::exception &ex) {
+        return fail(IDG_ERR_INVALID_ARG, ex.what());
+    }
+}
+
+idg_status idg_degrid_bands(const idg_plan *plan, const void *const *d_bands, int32_t nr_bands, int32_t band_rows,
+                            const float *d_uvw, const void *d_aterms, const float *d_taper, void *d_vis,
+                            idg_stream stream) {
+    try {
+        if (!plan) return fail(IDG_ERR_INVALID_ARG, "plan is NULL");
+        const cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+        if (plan->items.empty()) {   // every visibility dropped: all 0 (R-12, R-13)
+            const size_t bytes = size_t(plan->nr_baselines) * plan->nr_timesteps * plan->nr_channels * 32;
+            if (bytes > 0 && !d_vis) return fail(IDG_ERR_INVALID_ARG, "d_vis is NULL");
+            cudaError_t e = bytes > 0 ? cudaMemsetAsync(d_vis, 0, bytes, s) : cudaSuccess;
+            return e == cudaSuccess ? IDG_OK : cuda_fail(e, "cudaMemsetAsync(vis)");
+        }
+        idg_status st = validate_call(plan, d_vis, d_uvw, d_aterms, d_taper, d_bands);
+        if (st != IDG_OK) return st;
+        if ((st = validate_bands(plan, d_bands, nr_bands, band_rows)) != IDG_OK) return st;
+        const DeviceCopy *dc = nullptr;
+        if ((st = plan->device_copy(&dc)) != IDG_OK) return st;
+        cudaError_t e = zero_dropped(dc, d_vis, 0, 0, int64_t(plan->dropped.size() / 2), s);
+        if (e != cudaSuccess) return cuda_fail(e, "zero dropped visibilities");
+        idg::KernelArgs a = make_args(plan, dc, d_uvw, d_aterms, d_taper, d_vis, nullptr);
+        a.bands = reinterpret_cast<float2 *const *>(const_cast<void *const *>(d_bands));
+        a.band_rows = band_rows;
+        e = idg::launch_degridder(a, s);
+        if (e != cudaSuccess) return cuda_fail(e, "degridder launch (banded)");
+        return IDG_OK;
+    } catch (const std::exception &ex) {
+        return fail(IDG_ERR_INVALID_ARG, ex.what());
+    }
+}
+
+// CUDA IPC: a band allocated by one process, mapped into the others (peer access over NVLink / NVSwitch
+// enabled lazily by the driver).  Handles name whole allocations, so the pointer's offset inside its
+// allocation travels with the handle (cuMemGetAddressRange through the runtime's driver entry point: the
+// library does not link libcuda).
+using AddressRangeFn = int (*)(unsigned long long *, size_t *, unsigned long long);
+
+static cudaError_t allocation_base(const void *p, const void **base) {
+    static AddressRangeFn fn = nullptr;
+    if (!fn) {
+        void *f = nullptr;
+        cudaDriverEntryPointQueryResult q{};
+        cudaError_t e = cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q);
+        if (e != cudaSuccess) return e;
+        if (!f || q != cudaDriverEntryPointSuccess) return cudaErrorNotSupported;
+        fn = reinterpret_cast<AddressRangeFn>(f);
+    }
+    unsigned long long b = 0;
+    size_t n = 0;
+    if (fn(&b, &n, reinterpret_cast<unsigned long long>(p)) != 0) return cudaErrorInvalidValue;
+    *base = reinterpret_cast<const void *>(b);
+    return cudaSuccess;
+}
+
+idg_status idg_ipc_handle(const void *d_ptr, unsigned char handle[64], uint64_t *offset) {
+    if (!d_ptr || !handle || !offset) return fail(IDG_ERR_INVALID_ARG, "NULL argument");
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "CUDA IPC handle size");
+    const void *base = nullptr;
+    cudaError_t e = allocation_base(d_ptr, &base);
+    if (e != cudaSuccess) return cuda_fail(e, "allocation range of d_ptr");
+    cudaIpcMemHandle_t h;
+    if ((e = cudaIpcGetMemHandle(&h, const_cast<void *>(base))) != cudaSuccess) return cuda_fail(e, "cudaIpcGetMemHandle");
+    std::memcpy(handle, &h, 64);
+    *offset = uint64_t(static_cast<const char *>(d_ptr) - static_cast<const char *>(base));
+    return IDG_OK;
+}
+
+idg_status idg_ipc_open(const unsigned char handle[64], uint64_t offset, void **d_ptr) {
+    if (!handle || !d_ptr) return fail(IDG_ERR_INVALID_ARG, "NULL argument");
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle, 64);
+    void *base = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaIpcOpenMemHandle");
+    *d_ptr = static_cast<char *>(base) + offset;
+    return IDG_OK;
+}
+
+idg_status idg_ipc_close(void *d_ptr, uint64_t offset) {
+    if (!d_ptr) return fail(IDG_ERR_INVALID_ARG, "d_ptr is NULL");
+    cudaError_t e = cudaIpcCloseMemHandle(static_cast<char *>(d_ptr) - offset);
+    return e == cudaSuccess ? IDG_OK : cuda_fail(e, "cudaIpcCloseMemHandle");
+}
+
+// ------------------------------------------------------------------------------------------------
 // Host-streamed calls: the paper's asynchronous I/O with triple buffering (Fig. 7).  Work
 // groups (contiguous baseline ranges) stream through kStagingBuffers device buffers; uploads run on a
 // copy stream, downloads on another, kernels on the caller's stream, ordered with events.

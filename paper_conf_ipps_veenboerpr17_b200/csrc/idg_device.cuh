@@ -47,6 +47,27 @@ __device__ __forceinline__ void red_add(float2 *addr, float2 v) {
                  : "memory");
 }
 
+// Grid element (plane z, pol, row y, column x): in the device-resident grid, or -- banded grid -- in the band
+// of its owner, bands[y / R] (rows [r R, (r+1) R) of every [plane][pol], stored [planes][4][R][N]).
+__device__ __forceinline__ float2 *grid_elem(const KernelArgs &a, int z, int pol, int y, int x) {
+    if (a.bands) {
+        const int r = y / a.band_rows, ly = y - r * a.band_rows;
+        return a.bands[r] + ((int64_t(z) * 4 + pol) * a.band_rows + ly) * a.grid_size + x;
+    }
+    return a.grid + ((int64_t(z) * 4 + pol) * a.grid_size + y) * a.grid_size + x;
+}
+// The adder for one grid element.  Banded: the owner's band may be another GPU's memory (CUDA IPC over
+// NVLink / NVSwitch), so the sum uses scalar fp32 reductions, which peer memory supports everywhere.
+__device__ __forceinline__ void grid_add(const KernelArgs &a, int z, int pol, int y, int x, float2 v) {
+    float2 *p = grid_elem(a, z, pol, y, x);
+    if (a.bands) {
+        asm volatile("red.global.add.f32 [%0], %1;" ::"l"(&p->x), "f"(v.x) : "memory");
+        asm volatile("red.global.add.f32 [%0], %1;" ::"l"(&p->y), "f"(v.y) : "memory");
+    } else {
+        red_add(p, v);
+    }
+}
+
 // Centred-DFT twiddle table tw[r] = exp(sign 2 pi i r / N~), r = 0..N~-1 (R-5).
 template <int NS>
 __device__ __forceinline__ void init_twiddles(float2 *tw, float sign) {
@@ -191,9 +212,9 @@ __device__ __forceinline__ void gridder_epilogue(const KernelArgs &a, const Item
             a.subgrids[int64_t(blockIdx.x) * 4 * NPIX + o] = sum;
             continue;
         }
-        float2 *dst = a.grid + ((int64_t(md.z) * 4 + pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx;
-        red_add(dst, sum);
+        grid_add(a, md.z, pol, md.y + ky, md.x + kx, sum);
     }
+    if (a.bands) __threadfence_system();   // the peer-memory adds are visible before the kernel completes
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -208,7 +229,7 @@ __device__ __forceinline__ void degridder_split_columns(const KernelArgs &a, con
     for (int o = threadIdx.x; o < 4 * NPIX; o += nt) {
         const int pol = o / NPIX, rem = o - pol * NPIX, ky = rem / NS, kx = rem - ky * NS;
         sub_s[o] = a.subgrids ? a.subgrids[int64_t(blockIdx.x) * 4 * NPIX + o]   // host splitter
-                              : a.grid[((int64_t(md.z) * 4 + pol) * a.grid_size + md.y + ky) * a.grid_size + md.x + kx];
+                              : *grid_elem(a, md.z, pol, md.y + ky, md.x + kx);
     }
     init_twiddles<NS>(tw, +1.0f);
     __syncthreads();

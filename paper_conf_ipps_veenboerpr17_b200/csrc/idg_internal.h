@@ -49,6 +49,10 @@ struct KernelArgs {
     float2 *subgrids;            // nullptr, or [nr_items][4][N~][N~] in launch order: the gridders store their
                                  // transformed subgrids here instead of adding them to `grid`, the
                                  // degridders read their split subgrids from here (host adder / splitter)
+    float2 *const *bands;        // nullptr, or [nr_bands] pointers (banded grid, possibly peer memory of other
+                                 // ranks): grid rows [r R, (r+1) R) of every [plane][pol] live in bands[r] as
+                                 // [planes][4][R][N]; replaces `grid` (idg_grid_bands / idg_degrid_bands)
+    int32_t band_rows;           // R
     int32_t max_channels_in_item;
     int32_t max_timesteps_in_item;
     float mean_timesteps_in_item; // mean T~ over the items (short-item kernel choice)

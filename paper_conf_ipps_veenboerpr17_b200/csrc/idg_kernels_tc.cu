@@ -228,6 +228,13 @@ __device__ __forceinline__ void gridder_epilogue_tc(const KernelArgs &a, const I
         });
         return;
     }
+    if (a.bands) {   // banded grid: each element goes to its owner's band (peer memory)
+        dft_pass_tc<NS, WARPS>(tmp_s, NS, 1, tab, 1.0f, 32.0f / sc, [&](int pol, int kx, int ky, float2 v) {
+            dev::grid_add(a, md.z, pol, md.y + ky, md.x + kx, v);
+        });
+        __threadfence_system();
+        return;
+    }
     const int64_t gs = a.grid_size;
     float2 *gp = a.grid + (int64_t(md.z) * 4 * gs + md.y) * gs + md.x;
     dft_pass_tc<NS, WARPS>(tmp_s, NS, 1, tab, 1.0f, 32.0f / sc, [&](int pol, int kx, int ky, float2 v) {
@@ -257,7 +264,8 @@ __device__ __forceinline__ void degridder_prologue_tc(const KernelArgs &a, const
         const int o = threadIdx.x + i * NT;
         if (o < 4 * NPIX) {
             const int pol = o / NPIX, rem = o - pol * NPIX, ky = rem / NS, kx = rem - ky * NS;
-            v[i] = gp[(int64_t(pol) * gs + ky) * gs + kx];
+            v[i] = a.bands && !a.subgrids ? *dev::grid_elem(a, md.z, pol, md.y + ky, md.x + kx)   // owner's band
+                                          : gp[(int64_t(pol) * gs + ky) * gs + kx];
         }
     }
     dft_tab_to_smem<NS>(tab, +1);

@@ -458,6 +458,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kUrThreads, 2) gridd
                                                 });
             return;
         }
+        if (a.bands) {   // banded grid: each element goes to its owner's band (peer memory)
+            dft_pass_tc<NS, kUrThreads / 32, 2>(tmp_s, NS, 1, tab, 1.0f, 32.0f / sc,
+                                                [&](int pol, int kx, int ky, float2 v) {
+                                                    dev::grid_add(a, md.z, pol0 + pol, md.y + ky, md.x + kx, v);
+                                                });
+            __threadfence_system();
+            return;
+        }
         const int64_t gs = a.grid_size;
         float2 *gp = a.grid + (int64_t(md.z) * 4 * gs + md.y) * gs + md.x;
         dft_pass_tc<NS, kUrThreads / 32, 2>(tmp_s, NS, 1, tab, 1.0f, 32.0f / sc, [&](int pol, int kx, int ky, float2 v) {

@@ -49,6 +49,7 @@ EXPORTED = ["idg_plan_create", "idg_plan_destroy", "idg_plan_nr_subgrids", "idg_
             "idg_profiling_enable", "idg_profiling_reset", "idg_profiling_read", "idg_launch_count",
             "idg_kernel_variants", "idg_host_workspace_size", "idg_grid_host", "idg_degrid_host",
             "idg_host_adder_workspace_size", "idg_grid_host_adder", "idg_degrid_host_splitter",
+            "idg_grid_bands", "idg_degrid_bands", "idg_ipc_handle", "idg_ipc_open", "idg_ipc_close",
             "idg_status_string", "idg_last_error", "idg_last_variant"]
 
 
@@ -77,6 +78,11 @@ def lib() -> ctypes.CDLL:
     L.idg_host_adder_workspace_size.argtypes = [P, ctypes.POINTER(sz)]
     L.idg_grid_host_adder.argtypes = [P, P, P, P, P, P, P, sz, P]
     L.idg_degrid_host_splitter.argtypes = [P, P, P, P, P, P, P, sz, P]
+    L.idg_grid_bands.argtypes = [P, P, P, P, P, P, i32, i32, P]
+    L.idg_degrid_bands.argtypes = [P, P, i32, i32, P, P, P, P, P]
+    L.idg_ipc_handle.argtypes = [P, P, ctypes.POINTER(ctypes.c_uint64)]
+    L.idg_ipc_open.argtypes = [P, ctypes.c_uint64, ctypes.POINTER(P)]
+    L.idg_ipc_close.argtypes = [P, ctypes.c_uint64]
     for f in ("idg_rho_benchmark", "idg_rho_benchmark_scalar"):
         getattr(L, f).argtypes = [i32, i32, P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
     L.idg_profiling_enable.argtypes = [i32]
@@ -254,6 +260,64 @@ def degrid(plan: Plan, grid_in, uvw, aterms, taper, vis_out, stream=None):
     with _one_device(grid_in, uvw, aterms, taper, vis_out):
         _check(lib().idg_degrid(plan.handle, *args, None, 0, _stream(stream)), "idg_degrid")
     return vis_out
+
+
+def _bands_args(plan: Plan, bands_ptrs, band_rows: int):
+    """(device pointer array, count) of a banded grid: bands_ptrs is an int64 CUDA tensor of band pointers."""
+    import torch
+    if not (isinstance(bands_ptrs, torch.Tensor) and bands_ptrs.is_cuda and bands_ptrs.dtype == torch.int64
+            and bands_ptrs.dim() == 1 and bands_ptrs.is_contiguous()):
+        raise TypeError("bands_ptrs must be a contiguous 1-D int64 CUDA tensor of band pointers")
+    if band_rows < 1 or bands_ptrs.numel() * band_rows < plan.grid_size:
+        raise ValueError("the bands must cover the grid rows (nr_bands * band_rows >= grid_size)")
+    return ctypes.c_void_p(bands_ptrs.data_ptr()), int(bands_ptrs.numel())
+
+
+def grid_bands(plan: Plan, vis, uvw, aterms, taper, bands_ptrs, band_rows: int, stream=None):
+    """idg_grid_bands: every band += its rows of the gridded visibilities (the adder into the owners' bands,
+    possibly other ranks' memory: the cross-rank reduction fused into the gridder)."""
+    sh = _shapes(plan)
+    args = [_dev(vis, *sh["vis"], "vis"), _dev(uvw, *sh["uvw"], "uvw"), _dev(aterms, *sh["aterms"], "aterms"),
+            _dev(taper, *sh["taper"], "taper")]
+    bp, nb = _bands_args(plan, bands_ptrs, band_rows)
+    with _one_device(vis, uvw, aterms, taper, bands_ptrs):
+        _check(lib().idg_grid_bands(plan.handle, *args, bp, nb, int(band_rows), _stream(stream)), "idg_grid_bands")
+
+
+def degrid_bands(plan: Plan, bands_ptrs, band_rows: int, uvw, aterms, taper, vis_out, stream=None):
+    """idg_degrid_bands: vis_out = predictions from the banded model grid (the splitter reads the owners'
+    bands: no broadcast)."""
+    sh = _shapes(plan)
+    bp, nb = _bands_args(plan, bands_ptrs, band_rows)
+    args = [_dev(uvw, *sh["uvw"], "uvw"), _dev(aterms, *sh["aterms"], "aterms"), _dev(taper, *sh["taper"], "taper"),
+            _dev(vis_out, *sh["vis"], "vis")]
+    with _one_device(uvw, aterms, taper, vis_out, bands_ptrs):
+        _check(lib().idg_degrid_bands(plan.handle, bp, nb, int(band_rows), *args, _stream(stream)),
+               "idg_degrid_bands")
+    return vis_out
+
+
+def ipc_handle(t) -> tuple[bytes, int]:
+    """(64-byte CUDA IPC handle of t's allocation, byte offset of t in it)."""
+    h = (ctypes.c_ubyte * 64)()
+    off = ctypes.c_uint64(0)
+    with _one_device(t):
+        _check(lib().idg_ipc_handle(ctypes.c_void_p(t.data_ptr()), h, ctypes.byref(off)), "idg_ipc_handle")
+    return bytes(h), int(off.value)
+
+
+def ipc_open(handle: bytes, offset: int) -> int:
+    """Map another process's allocation (current device); returns the device pointer at `offset`."""
+    if len(handle) != 64:
+        raise ValueError("a CUDA IPC handle has 64 bytes")
+    p = ctypes.c_void_p()
+    _check(lib().idg_ipc_open((ctypes.c_ubyte * 64).from_buffer_copy(handle), ctypes.c_uint64(offset),
+                              ctypes.byref(p)), "idg_ipc_open")
+    return int(p.value)
+
+
+def ipc_close(ptr: int, offset: int):
+    _check(lib().idg_ipc_close(ctypes.c_void_p(ptr), ctypes.c_uint64(offset)), "idg_ipc_close")
 
 
 def _host(t, dtype, shape, name):

@@ -16,6 +16,11 @@ result is identical to the full-grid collective with less traffic.
 
 torch.distributed is plumbing only (NCCL over NVLink on B200, gloo for the CPU tests); every step of the
 hot path runs in libidg_b200.so.
+
+BandedGrid fuses both exchanges into the kernels instead: the grid is distributed by row bands (rank r owns
+rows [r R, (r+1) R) of every [plane][pol]), every rank's gridder adds each subgrid row straight into its
+owner's band through CUDA-IPC peer memory (NVLink / NVSwitch) and every degridder's splitter reads the
+owners' bands, so there is no reduce and no broadcast -- only a barrier between the two phases.
 """
 from __future__ import annotations
 
@@ -139,3 +144,119 @@ class ShardedIDG:
         from . import idg
         broadcast_grid(grid_in, src=src, rows=self.rows(grid_in.device))
         return idg.degrid_host(self.plan, grid_in, uvw, aterms, taper, vis_host_out, ws, stream=stream)
+
+
+# ---- banded grid: the exchange fused into the kernels (idg_grid_bands / idg_degrid_bands) --------------
+
+def band_rows(grid_size: int, world: int) -> int:
+    """Rows per band R = ceil(N / world): rank r owns grid rows [r R, min((r+1) R, N))."""
+    return -(-int(grid_size) // max(1, int(world)))
+
+
+def band_range(grid_size: int, world: int, rank: int):
+    R = band_rows(grid_size, world)
+    return min(rank * R, grid_size), min((rank + 1) * R, grid_size)
+
+
+def split_bands(full, world: int):
+    """The bands [..., R, N] of a full grid [..., N, N] (the last band zero-padded to R rows); numpy or torch."""
+    N = full.shape[-1]
+    R = band_rows(N, world)
+    out = []
+    for r in range(world):
+        y0, y1 = band_range(N, world, r)
+        if hasattr(full, "new_zeros"):
+            b = full.new_zeros(full.shape[:-2] + (R, N))
+        else:
+            b = np.zeros(full.shape[:-2] + (R, N), dtype=full.dtype)
+        b[..., : y1 - y0, :] = full[..., y0:y1, :]
+        out.append(b)
+    return out
+
+
+def join_bands(bands, grid_size: int):
+    """The full grid [..., N, N] from the bands (inverse of split_bands); numpy or torch."""
+    world = len(bands)
+    b0 = bands[0]
+    if hasattr(b0, "new_zeros"):
+        full = b0.new_zeros(b0.shape[:-2] + (grid_size, grid_size))
+    else:
+        full = np.zeros(b0.shape[:-2] + (grid_size, grid_size), dtype=b0.dtype)
+    for r, b in enumerate(bands):
+        y0, y1 = band_range(grid_size, world, r)
+        full[..., y0:y1, :] = b[..., : y1 - y0, :]
+    return full
+
+
+class BandedGrid:
+    """This rank's band of the distributed uv-grid plus peer mappings of every other rank's band.
+
+    Construction is collective (every rank of `group` must call it): the bands' CUDA-IPC handles are
+    exchanged once with all_gather_object and mapped (idg_ipc_open); `ptrs` is the device array of the
+    world's band pointers the kernels take.  Phases are separated by `sync()` (this rank's stream, then a
+    barrier): zero -> sync -> grid -> sync -> degrid (-> sync before the next zero)."""
+
+    def __init__(self, plan, device, group=None):
+        import torch
+        import torch.distributed as dist
+        from . import idg
+        self.plan, self.group = plan, group
+        on = dist.is_initialized() and dist.get_world_size(group) > 1
+        self.world = dist.get_world_size(group) if on else 1
+        self.rank = dist.get_rank(group) if on else 0
+        self.R = band_rows(plan.grid_size, self.world)
+        self.band = torch.zeros((plan.nr_w_planes, 4, self.R, plan.grid_size), dtype=torch.complex64, device=device)
+        self._opened = []
+        ptrs = [0] * self.world
+        ptrs[self.rank] = self.band.data_ptr()
+        if on:
+            handles = [None] * self.world
+            dist.all_gather_object(handles, idg.ipc_handle(self.band), group=group)
+            with torch.cuda.device(self.band.device):
+                for r, (h, off) in enumerate(handles):
+                    if r != self.rank:
+                        ptrs[r] = idg.ipc_open(h, off)
+                        self._opened.append((ptrs[r], off))
+        self.ptrs = torch.tensor(ptrs, dtype=torch.int64, device=device)
+
+    def sync(self, stream=None):
+        """This rank's queued work is complete and so is every other rank's (stream sync, then barrier)."""
+        import torch
+        import torch.distributed as dist
+        (torch.cuda.current_stream(self.band.device) if stream is None else stream).synchronize()
+        if self.world > 1:
+            dist.barrier(group=self.group)
+
+    def grid(self, vis, uvw, aterms, taper, stream=None):
+        """Add this rank's visibilities into the world's bands (idg_grid_bands)."""
+        from . import idg
+        idg.grid_bands(self.plan, vis, uvw, aterms, taper, self.ptrs, self.R, stream=stream)
+
+    def degrid(self, uvw, aterms, taper, vis_out, stream=None):
+        """Predict this rank's visibilities from the world's bands (idg_degrid_bands)."""
+        from . import idg
+        return idg.degrid_bands(self.plan, self.ptrs, self.R, uvw, aterms, taper, vis_out, stream=stream)
+
+    def gather(self, dst: int = 0):
+        """The full grid [nz][4][N][N] on rank `dst` (None elsewhere) -- for checks and the image step."""
+        import torch.distributed as dist
+        N = self.plan.grid_size
+        if self.world == 1:
+            return join_bands([self.band], N)
+        parts = [None] * self.world if self.rank == dst else None
+        dist.gather_object(self.band.cpu(), parts, dst=dst, group=self.group)
+        return join_bands([p.to(self.band.device) for p in parts], N) if self.rank == dst else None
+
+    def load(self, full):
+        """Set this rank's band from a full grid [nz][4][N][N] (or [4][N][N]) every rank holds."""
+        N = self.plan.grid_size
+        y0, y1 = band_range(N, self.world, self.rank)
+        f = full.reshape(self.band.shape[:2] + (N, N))
+        self.band.zero_()
+        self.band[:, :, : y1 - y0, :] = f[:, :, y0:y1, :]
+
+    def close(self):
+        from . import idg
+        for p, off in self._opened:
+            idg.ipc_close(p, off)
+        self._opened = []

@@ -14,17 +14,20 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 @pytest.mark.gpu
-def test_two_rank_bench_on_one_gpu(tmp_path):
+@pytest.mark.parametrize("exchange,port", [("nccl", 29547), ("peer", 29548)])
+def test_two_rank_bench_on_one_gpu(exchange, port, tmp_path):
     env = dict(os.environ, IDG_BENCH_SHARED_GPU="1")
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
-           "--master-addr", "127.0.0.1", "--master-port", "29547", os.path.join(ROOT, "bench.py"),
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"),
            "--gpus", "2", "--config", "lofar", "--steps", "2", "--warmup", "3", "--timesteps", "512",
-           "--e2e-steps", "2", "--no-cpu-baseline", "--rho-iterations", "256", "--no-rho-sweep", "--no-kernel-energy"]
+           "--e2e-steps", "2", "--no-cpu-baseline", "--rho-iterations", "256", "--no-rho-sweep", "--no-kernel-energy",
+           "--exchange", exchange]
     p = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=900)
     assert p.returncode == 0, p.stderr[-3000:]
     lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
     assert len(lines) == 1, p.stdout[-2000:]
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["gpu_launches"] > 0
+    assert ("banded" in d["config"]["parallelism"]) == (exchange == "peer")
     assert d["e2e"]["value"] > 0
     assert d["e2e"]["check"]["adjoint_identity_rel_err"] < 1e-4
