@@ -408,6 +408,20 @@ def run_ours(args):
         energy = {"J_per_step": joules / args.steps, "avg_W": joules / (ms * 1e-3),
                   "GOps_per_J": ops / joules / 1e9, "source": "NVML total energy counter, this GPU, timed region"}
 
+    # ---- roofline denominators, measured right after the timed region on an idle GPU (before the host-
+    # streamed legs: measured after them, the rho = 17 kernel ran 15-40% slow in some runs, r02y) ----------
+    def best(rho, iters, scalar=False):
+        return max(idg.rho_benchmark(rho, iters, scalar=scalar)[0] for _ in range(5))
+    barrier()
+    with ClockSampler(local) as rclocks:
+        sincos_per_s = best(0, 4 * args.rho_iterations) / 2.0
+        rho17 = best(17, args.rho_iterations) / 1e12
+        rho17_scalar = best(17, args.rho_iterations, scalar=True) / 1e12
+        rho_sweep = {}
+        if not args.no_rho_sweep:
+            for r in (0, 1, 2, 4, 8, 12, 16, 17, 24, 32, 64):
+                rho_sweep[str(r)] = best(r, args.rho_iterations) / 1e12
+
     # ---- energy per kernel (Fig. 15: GFlops/W of the gridder and the degridder) -----------
     # separate timed loops of one kernel each, NVML board energy over the loop
     if energy is not None and not args.no_kernel_energy:
@@ -473,17 +487,6 @@ def run_ours(args):
                                            world, rank, nvis_total, bufs, grid_d, sharded, barrier, inplace)
     bufs.clear()
 
-    # ---- roofline ---------------------------------------------------------------------------------
-    def best(rho, iters, scalar=False):
-        return max(idg.rho_benchmark(rho, iters, scalar=scalar)[0] for _ in range(3))
-    with ClockSampler(local) as rclocks:
-        sincos_per_s = best(0, 4 * args.rho_iterations) / 2.0
-        rho17 = best(17, args.rho_iterations) / 1e12
-        rho17_scalar = best(17, args.rho_iterations, scalar=True) / 1e12
-        rho_sweep = {}
-        if not args.no_rho_sweep:
-            for r in (0, 1, 2, 4, 8, 12, 16, 17, 24, 32, 64):
-                rho_sweep[str(r)] = best(r, args.rho_iterations) / 1e12
     xu_peak = sincos_per_s * OPS_PER_PAIR / 1e12
     per_kernel = {}
     for name in ("gridder", "degridder"):

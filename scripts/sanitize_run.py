@@ -14,7 +14,8 @@ import numpy as np  # noqa: E402
 
 import idgsynth  # noqa: E402
 
-FAMILIES = {"default": (None, None), "tc": ("tc", "tc"), "simt": ("simt", "simt")}
+FAMILIES = {"default": (None, None), "tc": ("tc", "tc"), "simt": ("simt", "simt"),
+            "umma": ("gridder_umma_rot<*", "")}
 
 
 def main():
@@ -22,6 +23,8 @@ def main():
     kw = {}
     if name == "ska_small":
         name, kw = "ska", dict(T=128, nr_stations=3)
+    if name == "predict_small":       # 16-channel items at N~ = 32 (the KPT 2 rotation / tcgen05 gridders)
+        name, kw = "predict", dict(T=128, nr_stations=3)
     if name == "lofar_small":
         name, kw = "lofar", dict(T=256, nr_stations=4)
     if name == "small_dde8":          # 8 channels: the N~ = 16 rotation gridder (KPT 1) and 8-row degridder
@@ -58,6 +61,13 @@ def main():
     gh = torch.zeros(shape, dtype=torch.complex64)
     idg.grid_host_adder(plan, vh, uvw, at, tp, gh, wa)
     idg.degrid_host_splitter(plan, gh, uvw, at, tp, out, wa)
+    # the banded grid (3 bands in separate allocations): adder into / splitter from the owners' bands
+    from paper_conf_ipps_veenboerpr17_b200 import parallel
+    R = parallel.band_rows(obs.grid_size, 3)
+    bands = [torch.zeros(shape[:-2] + (R, obs.grid_size), dtype=torch.complex64, device="cuda") for _ in range(3)]
+    ptrs = torch.tensor([b.data_ptr() for b in bands], dtype=torch.int64, device="cuda")
+    idg.grid_bands(plan, dev(vis), uvw, at, tp, ptrs, R)
+    idg.degrid_bands(plan, ptrs, R, uvw, at, tp, V)
     torch.cuda.synchronize()
     print(f"sanitize_run {name} {fam}: {plan.nr_subgrids} items, gridder {idg.last_variant('gridder')}, "
           f"degridder {idg.last_variant('degridder')}, launches {idg.launch_count()}")
