@@ -72,6 +72,9 @@ CASES = [
     ("small_dde", dict(C=64), None, "spheroidal"),                   # 2 blocks of 32 channels per timestep
     ("small_dde", dict(C=40, C_block=24), None, "spheroidal"),      # 24 + 16 channels: mixed item widths
     ("lofar", dict(T=256, nr_stations=5, channels="gap_jitter"), None, "asymmetric"),  # real channel table
+    ("tiny", dict(T=1), "identity", "asymmetric"),                   # degenerate: one timestep, one channel
+    ("small_dde", dict(nr_stations=2), None, "asymmetric"),          # degenerate: a single baseline
+    ("small_dde", dict(T=1, C=1), None, "spheroidal"),              # one visibility per baseline
 ]
 
 
