@@ -1,5 +1,6 @@
 """C-ABI library (no GPU): it loads, exports every function include/idg.h declares, validates its
 arguments, and its host plan builder is bit-exact with the oracle's plan (R-8..R-16)."""
+import ctypes
 import dataclasses
 import os
 import re
@@ -119,3 +120,26 @@ def test_calls_on_a_plan_without_items_need_no_gpu():
     assert not vis.any()
     assert lib.idg_grid_host(h, None, None, None, None, None, None, 0, None) == 0      # nothing to add
     assert lib.idg_grid(h, None, None, None, None, None, None, 0, None) == 0
+
+
+def test_banded_and_ipc_calls_validate_arguments_without_a_gpu():
+    """The banded-grid and IPC entry points reject bad arguments before touching the device."""
+    obs = idgsynth.make_observation("small_dde")
+    plan = idg.Plan.from_observation(obs)
+    lib = idg.lib()
+    h = plan._h
+    fake = ctypes.c_void_p(0x1000)   # never dereferenced: validation fails first
+    # NULL bands / bands that do not cover the grid rows
+    assert lib.idg_grid_bands(h, fake, fake, fake, fake, None, 1, obs.grid_size, None) == 1
+    assert "d_bands" in lib.idg_last_error().decode()
+    assert lib.idg_grid_bands(h, fake, fake, fake, fake, fake, 2, obs.grid_size // 2 - 1, None) == 1
+    assert "cover" in lib.idg_last_error().decode()
+    assert lib.idg_grid_bands(h, fake, fake, fake, fake, fake, 0, obs.grid_size, None) == 1
+    assert lib.idg_degrid_bands(h, None, 1, obs.grid_size, fake, fake, fake, fake, None) == 1
+    assert lib.idg_degrid_bands(h, fake, 3, 1, fake, fake, fake, fake, None) == 1
+    assert lib.idg_grid_bands(None, fake, fake, fake, fake, fake, 1, obs.grid_size, None) == 1
+    # IPC: NULL arguments
+    off = ctypes.c_uint64()
+    assert lib.idg_ipc_handle(None, (ctypes.c_ubyte * 64)(), ctypes.byref(off)) == 1
+    assert lib.idg_ipc_open(None, 0, ctypes.byref(ctypes.c_void_p())) == 1
+    assert lib.idg_ipc_close(None, 0) == 1
