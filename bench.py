@@ -217,12 +217,15 @@ def sincos_per_pair(variant: str, nc_item: int) -> float:
     """sincos evaluations per (pixel, visibility) pair of a kernel variant (the paper's kernels and the
     direct tensor-core kernels: 1).  gridder_rot2: per (pixel, timestep) the 8 group-0 slot phasors for
     8 J pairs (J = channel groups of 8; E_t is derived from them); degridder_rot / rot8 / rot16: per
-    (visibility row 0, pixel) one phasor and one rotation E for 4 / 8 / 16 channel rows."""
+    (visibility row 0, pixel) one phasor and one rotation E for 4 / 8 / 16 channel rows (rot16s2: plus the
+    phasor of row 8, which starts the second rotation chain)."""
     j = max(1, nc_item // 8)
     if variant.startswith("gridder_rot2"):
         return 1.0 / j
     if variant.startswith("gridder_rot"):
         return (8.0 + (4.0 if j > 1 else 0.0)) / (8.0 * j)
+    if variant.startswith("degridder_rot16s2"):
+        return 3.0 / 16      # row 0, E and row 8 (the second rotation chain's start)
     if variant.startswith("degridder_rot16"):
         return 2.0 / 16
     if variant.startswith("degridder_rot8"):

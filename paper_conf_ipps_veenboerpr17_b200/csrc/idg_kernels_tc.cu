@@ -80,6 +80,36 @@ __device__ __forceinline__ void split2(float x, float y, uint32_t &hi, uint32_t 
 }
 __device__ __forceinline__ void split_phasor(float x, float y, uint32_t &hi, uint32_t &lo) { split2(x, y, hi, lo); }
 
+// Fixed-point phasor split by byte permutation (the degridders' A operand; scripts/split_probe.cu).
+// W = fl(sigma z + M) with M = 2^23 + 0x680000 + 2^17 is an fp32 in [2^23, 2^24) (ulp 1), so its bits are
+// 0x4B | 0x68 + (X >> 16) | X >> 8 | X (bytes 3..0) with X = 2^17 + rn(sigma z) in [0, 2^18) for |z| <= 1.
+// Read as f16: bytes (1, 2) = 2048 + 2 (X >> 8) (binade [2048, 4096), ulp 2) and bytes (0, 3) =
+// 14 + (X & 255) / 128 (binade [8, 16), ulp 1/128), so hi + lo = 2062 + X / 128 = kFxOffset + kFxGain z_q
+// exactly, z_q = rn(sigma z) / sigma (|z - z_q| <= 2^-18).  One FFMA2 per packed pair + two PRMT per
+// phasor replace F2FP + 2 FHFMA + F2FP.  The products hi*(B_hi + B_lo) + lo*B_hi then carry
+// kFxOffset * sum_k B_k + kFxLo * sum_k B_lo,k per output column (the same for every visibility), removed
+// in the epilogue (degridder_setup_tc computes the column sums); lo*B_lo beyond its constant part is
+// <= 2 |B_lo| per term (2^-20 of a term) and dropped.
+constexpr float kFxSigma = 130944.0f;     // 2^17 - 128: gain sigma / 128 = 1023
+constexpr float kFxMagic = 15335424.0f;   // 2^23 + 0x680000 + 2^17
+constexpr float kFxOffset = 3086.0f;      // 2062 + 2^17 / 128
+constexpr float kFxLo = 14.0f;            // constant part of lo
+constexpr float kFxGain = 1023.0f;
+__device__ __forceinline__ uint32_t prmt(float a, float b, uint32_t sel) {
+    uint32_t r;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(__float_as_uint(a)), "r"(__float_as_uint(b)), "r"(sel));
+    return r;
+}
+// C = (cos, cos), S = (sin, sin) of the phasors at k-slots q and q+4 (packed): their A registers.
+__device__ __forceinline__ void split_fx(f2p C, f2p S, uint32_t &hq, uint32_t &lq, uint32_t &hq4, uint32_t &lq4) {
+    const float2 w = unpk(fma2(C, dup(kFxSigma), dup(kFxMagic)));
+    const float2 v = unpk(fma2(S, dup(kFxSigma), dup(kFxMagic)));
+    hq = prmt(w.x, v.x, 0x6521);
+    lq = prmt(w.x, v.x, 0x7430);
+    hq4 = prmt(w.y, v.y, 0x6521);
+    lq4 = prmt(w.y, v.y, 0x7430);
+}
+
 
 __device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
                                          uint32_t b0, uint32_t b1) {
@@ -864,9 +894,11 @@ struct DegridSmem {
 // Degridder prologue shared by the tensor-core degridders: per-timestep phase coefficients, a6 + a7
 // (tensor-core DFT), a8 per pixel, and the corrected subgrid as split B fragments (k-block = 8 pixels)
 // + per-pixel {l, m, n}.  Ends with a barrier; returns 1 / (the power-of-two f16 range scale).
+// off_s (optional, [8 (WARPS + 1)], the tail is scratch): per B column n, kFxOffset * sum_k (B_hi + B_lo)[k][n] - kFxLo * sum_k B_lo[k][n]
+// over the item's K rows -- the constant the fixed-point A operand adds to every output of column n.
 template <int NS, int WARPS>
 __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const ItemSetup &s, const DegridSmem<NS> &sm,
-                                                    float *red_s) {
+                                                    float *red_s, float *off_s = nullptr) {
     constexpr int NT = WARPS * 32;
     constexpr int NPIX = NS * NS;
     constexpr int PPT = (NPIX + NT - 1) / NT;
@@ -909,6 +941,9 @@ __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const I
     }
     const float scale = pow2_scale(block_max<WARPS>(mx, red_s));  // barriers: sub_s reads are done
     uint32_t *frag_w = reinterpret_cast<uint32_t *>(sm.frag_s);
+    float colb[8], coll[8];   // this thread's part of the column sums of B_hi + B_lo and of B_lo (off_s)
+#pragma unroll
+    for (int gg = 0; gg < 8; ++gg) colb[gg] = coll[gg] = 0.0f;
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
         const int pix = threadIdx.x + i * NT;
@@ -924,7 +959,30 @@ __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const I
                 const int e = (kb * 32 + gg * 4 + qq) * 4;
                 frag_w[e + half] = hi;
                 frag_w[e + 2 + half] = lo;
+                if (off_s) {
+                    const float2 fh = __half22float2(*reinterpret_cast<const __half2 *>(&hi));
+                    const float2 fl = __half22float2(*reinterpret_cast<const __half2 *>(&lo));
+                    coll[gg] += fl.x + fl.y;
+                    colb[gg] += (fh.x + fh.y) + (fl.x + fl.y);
+                }
             }
+        }
+    }
+    if (off_s) {
+        // deterministic block sums of the column partials: warp shuffles, then per-warp rows off_s[8 + 8 w]
+        // summed in warp order
+#pragma unroll
+        for (int gg = 0; gg < 8; ++gg) {
+            float v = kFxOffset * colb[gg] - kFxLo * coll[gg];
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+            if ((threadIdx.x & 31) == 0) off_s[8 + 8 * (threadIdx.x >> 5) + gg] = v;
+        }
+        __syncthreads();
+        if (threadIdx.x < 8) {
+            float v = 0.0f;
+            for (int w = 0; w < WARPS; ++w) v += off_s[8 + 8 * w + threadIdx.x];
+            off_s[threadIdx.x] = v;
         }
     }
     __syncthreads();
@@ -942,13 +1000,16 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
     const float *df_s = sm.df_s;
     __shared__ float red_s[WARPS];
+    __shared__ float off_s[8 * (WARPS + 1)];
 
     const int item = a.order[blockIdx.x];
     const ItemSetup s = dev::item_setup(a, item, NS);
     const idg_metadata &md = s.md;
     const int nc = s.nc;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
-    const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s);
+    // fixed-point A operand (split_fx): output = (acc - column offset) * inv
+    const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s, off_s) * (1.0f / kFxGain);
+    const float off0 = off_s[2 * q], off1 = off_s[2 * q + 1];
 
     const int nvis = md.nr_timesteps * nc;
     const int ntiles = (nvis + 15) >> 4;
@@ -1000,8 +1061,8 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
                 __sincosf(p0.y, &sn[2], &cs[2]);  // row g,   slot q+4
                 __sincosf(p1.x, &sn[1], &cs[1]);  // row g+8, slot q
                 __sincosf(p1.y, &sn[3], &cs[3]);  // row g+8, slot q+4
-#pragma unroll
-                for (int j = 0; j < 4; ++j) split_phasor(cs[j], sn[j], ah[i][j], al[i][j]);
+                split_fx(pk(cs[0], cs[1]), pk(sn[0], sn[1]), ah[i][0], al[i][0], ah[i][1], al[i][1]);
+                split_fx(pk(cs[2], cs[3]), pk(sn[2], sn[3]), ah[i][2], al[i][2], ah[i][3], al[i][3]);
             }
 #pragma unroll
             for (int i = 0; i < MT; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
@@ -1017,7 +1078,8 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
                 const int v = (tile0 + i) * 16 + g + 8 * r;
                 if (v < nvis) {
                     const int t = tstep(v), c = v - t * nc;
-                    vis0[int64_t(t) * row + c * 4 + q] = make_float2(acc[i][2 * r] * inv, acc[i][2 * r + 1] * inv);
+                    vis0[int64_t(t) * row + c * 4 + q] =
+                        make_float2((acc[i][2 * r] - off0) * inv, (acc[i][2 * r + 1] - off1) * inv);
                 }
             }
         }
@@ -1039,7 +1101,9 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 // sincos pair per k-block (measured: N~ = 32 SKA 2140 -> 2186 MVis/s, predict +0.5%; N~ = 24 LOFAR -3.7%,
 // so it is the default for N~ = 32 only).  A one-tile software pipeline of the HMMAs (tried as SCH = 1)
 // compiles to the same SASS as 0: ptxas already spaces the HMMAs 5-12 instructions apart.
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int SCH = 0>
+// FX: the A operand split.  1 (default): fixed-point split by byte permutation (split_fx; N~ = 32 SKA loop
+// 7.8 -> 8.8 pairs/clk/SM in scripts/split_probe.cu); 0: the f16 hi/lo split (split2).
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int SCH = 0, int FX = 1>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
     constexpr int NKB = NPIX / 8;
@@ -1049,13 +1113,26 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
     const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
     const float *df_s = sm.df_s;
     __shared__ float red_s[WARPS];
+    __shared__ float off_s[FX ? 8 * (WARPS + 1) : 1];
 
     const int item = a.order[blockIdx.x];
     const ItemSetup s = dev::item_setup(a, item, NS);
     const idg_metadata &md = s.md;
     const int nc = s.nc;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
-    const float inv = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s);
+    const float inv0 = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s, FX ? off_s : nullptr);
+    // output = (acc - off) inv: the fixed-point operand's gain and per-column offset removed
+    const float inv = FX ? inv0 * (1.0f / kFxGain) : inv0;
+    const float off0 = FX ? off_s[2 * q] : 0.0f, off1 = FX ? off_s[2 * q + 1] : 0.0f;
+    auto split = [](f2p C, f2p S, uint32_t &hq, uint32_t &lq, uint32_t &hq4, uint32_t &lq4) {
+        if constexpr (FX) {
+            split_fx(C, S, hq, lq, hq4, lq4);
+        } else {
+            const float2 cc = unpk(C), ss = unpk(S);
+            split_phasor(cc.x, ss.x, hq, lq);
+            split_phasor(cc.y, ss.y, hq4, lq4);
+        }
+    };
 
     // A warp unit is 8 R visibilities = R channel rows (stride CS) for each of the 8 lane groups g, as R / 2
     // m-tiles (lane group g owns rows g and g+8 of every tile):
@@ -1118,10 +1195,8 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                         S = fma2(C, ES, mul2(S, EC));
                         C = Cn;
                     }
-                    const float2 cc = unpk(C), ss = unpk(S);
                     // tile r >> 1, row g (r even) / g+8 (r odd): A regs {(row, q), (row+8, q), (row, q+4), (row+8, q+4)}
-                    split_phasor(cc.x, ss.x, ah[r >> 1][r & 1], al[r >> 1][r & 1]);
-                    split_phasor(cc.y, ss.y, ah[r >> 1][2 + (r & 1)], al[r >> 1][2 + (r & 1)]);
+                    split(C, S, ah[r >> 1][r & 1], al[r >> 1][r & 1], ah[r >> 1][2 + (r & 1)], al[r >> 1][2 + (r & 1)]);
                 }
 #pragma unroll
                 for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
@@ -1151,11 +1226,8 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                             S2 = fma2(C2, ES, mul2(S2, EC));
                             C2 = Cm;
                         }
-                        const float2 cc = unpk(C), ss = unpk(S), cc2 = unpk(C2), ss2 = unpk(S2);
-                        split_phasor(cc.x, ss.x, ah[h2], al[h2]);
-                        split_phasor(cc.y, ss.y, ah[2 + h2], al[2 + h2]);
-                        split_phasor(cc2.x, ss2.x, bh[h2], bl[h2]);
-                        split_phasor(cc2.y, ss2.y, bh[2 + h2], bl[2 + h2]);
+                        split(C, S, ah[h2], al[h2], ah[2 + h2], al[2 + h2]);
+                        split(C2, S2, bh[h2], bl[h2], bh[2 + h2], bl[2 + h2]);
                     }
                     mma3(acc[i], ah, al, bf);
                     mma3(acc[i + H], bh, bl, bf);
@@ -1172,9 +1244,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                             S = fma2(C, ES, mul2(S, EC));
                             C = Cn;
                         }
-                        const float2 cc = unpk(C), ss = unpk(S);
-                        split_phasor(cc.x, ss.x, ah[h2], al[h2]);
-                        split_phasor(cc.y, ss.y, ah[2 + h2], al[2 + h2]);
+                        split(C, S, ah[h2], al[h2], ah[2 + h2], al[2 + h2]);
                     }
                     mma3(acc[i], ah, al, bf);
                 }
@@ -1184,7 +1254,8 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
             float2 *vt = vis0 + int64_t(t) * row + int64_t(c0) * 4 + q;
 #pragma unroll
             for (int r = 0; r < R; ++r)
-                vt[r * CS * 4] = make_float2(acc[r >> 1][2 * (r & 1)] * inv, acc[r >> 1][2 * (r & 1) + 1] * inv);
+                vt[r * CS * 4] = make_float2((acc[r >> 1][2 * (r & 1)] - off0) * inv,
+                                             (acc[r >> 1][2 * (r & 1) + 1] - off1) * inv);
         }
     }
 }
@@ -1285,9 +1356,9 @@ template <int NS, int WARPS, int MT, int MINB>
 cudaError_t launch_degridder_tc(const KernelArgs &a, cudaStream_t st) {
     return launch_tc(degridder_tc_kernel<NS, WARPS, MT, MINB>, "degridder", smem_degridder_tc<NS>(a), WARPS * 32, a, st);
 }
-template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int SCH = 0>
+template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int SCH = 0, int FX = 1>
 cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
-    return launch_tc(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R, SCH>, "degridder", smem_degridder_tc<NS>(a),
+    return launch_tc(degridder_rot_kernel<NS, WARPS, MINB, UNR, CPT, R, SCH, FX>, "degridder", smem_degridder_tc<NS>(a),
                      WARPS * 32, a, st);
 }
 
@@ -1355,7 +1426,7 @@ const Variant kTcGridder[] = {
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>, 0, \
      smem_degridder_tc<NS>}
 const Variant kTcDegridder[] = {
-    TDROTS(24, 4, 3, 2, 16, 8), TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 1, 32, 16, 2),
+    TDROTS(24, 4, 3, 2, 16, 8), TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 2, 32, 16, 2),
     TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
     TDROTC(24, 8, 2, 1, 8, 8, "degridder_rot8"), TDROTC(32, 16, 2, 1, 8, 8, "degridder_rot8"),
@@ -1368,6 +1439,11 @@ const Variant kTcDegridder[] = {
     // items) -- selected by name only
     TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"),
     TDROTC(24, 8, 2, 1, 16, 8, "degridder_rot8"),
+    // the f16 hi/lo operand split (the default before the fixed-point split), for measurement
+    {24, 16, kTensor, 1, "degridder_rot16f<24,W4,minB3,U4,C16>", launch_degridder_rot<24, 4, 3, 4, 16, 16, 0, 0>, 16,
+     smem_degridder_tc<24>},
+    {32, 32, kTensor, 1, "degridder_rot16s2f<32,W8,minB2,U1,C32>", launch_degridder_rot<32, 8, 2, 1, 32, 16, 2, 0>, 32,
+     smem_degridder_tc<32>},
 };
 #undef TDROTC
 #undef TDROTS

@@ -19,6 +19,7 @@ def test_sincos_per_pair_by_family():
     assert spp("degridder_rot<24,W8,minB4,U1,C16>", 16) == 0.5       # row 0 + E for 4 rows
     assert spp("degridder_rot8<24,W8,minB2,U1,C16>", 16) == 0.25
     assert spp("degridder_rot16<24,W4,minB3,U4,C16>", 16) == 0.125
+    assert spp("degridder_rot16s2<32,W8,minB2,U2,C32>", 32) == 0.1875  # + row 8 (second chain)
 
 
 def test_ops_per_pair_is_the_papers():
