@@ -110,6 +110,46 @@ __device__ __forceinline__ void split_fx(f2p C, f2p S, uint32_t &hq, uint32_t &l
     lq4 = prmt(w.y, v.y, 0x7430);
 }
 
+// Integer tensor-core form of the degridder contraction (FX = 2; scripts/split_probe.cu "IMMA").  A phasor
+// component z becomes the 16-bit offset fixed-point X = 2^15 + rn(sigma z) held in the low half of
+// W = fl(sigma z + 2^23 + 2^15) (fp32 in [2^23, 2^24): ulp 1), i.e. two u8 limbs a_l = X & 255, a_h = X >> 8;
+// one PRMT gathers (c_l, c_h, s_l, s_h) of a phasor into the A register of mma.m16n8k32 (u8), one FFMA2
+// per packed pair forms W.  The corrected subgrid value x (24-bit signed fixed point, per-item power-of-two
+// scale) is three signed-digit s8 limbs x = 2^16 x_h + 2^8 x_m + x_l, and A x = 2^24 a_h x_h +
+// 2^16 (a_l x_h + a_h x_m) + 2^8 (a_l x_m + a_h x_l) + a_l x_l: one s32-accumulated mma per weight class
+// (B bytes (0, x_h), (x_h, x_m), (x_m, x_l) against (a_l, a_h)), a_l x_l (<= 2^-24 of a term) dropped.
+// Integer products and sums are exact; the offset 2^15 sum_k x_k per output column is removed in the
+// epilogue.  One PRMT per phasor (the f16 forms need two: the hi and the lo register).
+constexpr float kI8Sigma = 32767.0f;
+constexpr float kI8Magic = 8421376.0f;    // 2^23 + 2^15
+__device__ __forceinline__ void split_i8(f2p C, f2p S, uint32_t &aq, uint32_t &aq4) {
+    const float2 w = unpk(fma2(C, dup(kI8Sigma), dup(kI8Magic)));
+    const float2 v = unpk(fma2(S, dup(kI8Sigma), dup(kI8Magic)));
+    aq = prmt(w.x, v.x, 0x5410);
+    aq4 = prmt(w.y, v.y, 0x5410);
+}
+__device__ __forceinline__ void imma16832(int (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+    asm("mma.sync.aligned.m16n8k32.row.col.s32.u8.s8.s32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, {%0,%1,%2,%3};"
+        : "+r"(d[0]), "+r"(d[1]), "+r"(d[2]), "+r"(d[3]) : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+// The three weight classes of one tile; bf = {(x_h, x_m) limbs of slots q, q+4, (x_m, x_l) limbs of slots
+// q, q+4}, the (0, x_h) class derived from the first by a byte permutation.
+__device__ __forceinline__ void imma3(int (&d)[3][4], const uint32_t (&a)[4], const uint4 &bf, uint32_t h0, uint32_t h1) {
+    imma16832(d[0], a, h0, h1);
+    imma16832(d[1], a, bf.x, bf.y);
+    imma16832(d[2], a, bf.z, bf.w);
+}
+__device__ __forceinline__ uint32_t i8_high_limbs(uint32_t w16) {
+    uint32_t r;
+    asm("prmt.b32 %0, %1, 0, 0x2404;" : "=r"(r) : "r"(w16));
+    return r;
+}
+// (2^24 d0 + 2^16 d1 + 2^8 d2 - off) inv, exact in fp64 up to the final product
+__device__ __forceinline__ float i8_out(const int (&d)[3][4], int j, double off, double inv) {
+    const double t = fma(double(d[0][j]), 16777216.0, fma(double(d[1][j]), 65536.0, double(d[2][j]) * 256.0));
+    return float((t - off) * inv);
+}
+
 
 __device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
                                          uint32_t b0, uint32_t b1) {
@@ -896,7 +936,10 @@ struct DegridSmem {
 // + per-pixel {l, m, n}.  Ends with a barrier; returns 1 / (the power-of-two f16 range scale).
 // off_s (optional, [8 (WARPS + 1)], the tail is scratch): per B column n, kFxOffset * sum_k (B_hi + B_lo)[k][n] - kFxLo * sum_k B_lo[k][n]
 // over the item's K rows -- the constant the fixed-point A operand adds to every output of column n.
-template <int NS, int WARPS>
+// BM = 1: the B fragments as the s8 limbs of the integer form (FX = 2) instead: per (k-block, lane)
+// {(x_h, x_m) of slot q, of q+4, (x_m, x_l) of slot q, of q+4}; off_s (16-byte aligned, 16 (WARPS + 1) + 8
+// floats) gets 2^15 sum_k x[k][n] as doubles at double index 8 WARPS + n; returns 1 / (scale sigma).
+template <int NS, int WARPS, int BM = 0>
 __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const ItemSetup &s, const DegridSmem<NS> &sm,
                                                     float *red_s, float *off_s = nullptr) {
     constexpr int NT = WARPS * 32;
@@ -938,6 +981,64 @@ __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const I
             rec[4 + half] = dev::w_term_n(l, m);
             rec[6 + half] = 0.0f;
         }
+    }
+    if constexpr (BM == 1) {
+        // integer limbs: x = rn(value * scale) with max |x| in [2^21, 2^22) (power of two: exact scaling)
+        const float bmx = block_max<WARPS>(mx, red_s);
+        float scale = 1.0f;
+        if (bmx > 0.0f) {
+            const int e = int((__float_as_uint(bmx) >> 23) & 0xff) - 127;
+            scale = __uint_as_float(uint32_t(127 + min(max(21 - e, -120), 120)) << 23);
+        }
+        uint32_t *frag_w = reinterpret_cast<uint32_t *>(sm.frag_s);
+        double colx[8];
+#pragma unroll
+        for (int gg = 0; gg < 8; ++gg) colx[gg] = 0.0;
+        auto limbs = [](int x, int &h, int &m, int &l) {   // signed digits, x = 2^16 h + 2^8 m + l
+            l = ((x + 128) & 255) - 128;
+            const int y = (x - l) >> 8;
+            m = ((y + 128) & 255) - 128;
+            h = (y - m) >> 8;
+        };
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) {
+            const int pix = threadIdx.x + i * NT;
+            if (pix < NPIX) {
+                const int kb = pix >> 3, slot = pix & 7, qq = slot & 3, half = slot >> 2;
+#pragma unroll
+                for (int gg = 0; gg < 8; ++gg) {
+                    const int pol = gg >> 1;
+                    const int xr = __float2int_rn(rr[i][pol].x * scale), xi = __float2int_rn(rr[i][pol].y * scale);
+                    // column 2pol: (cos, sin) rows -> (Sre, Sim); column 2pol+1 -> (Sim, -Sre)
+                    const int xc = (gg & 1) ? xi : xr, xs = (gg & 1) ? -xr : xi;
+                    int ch, cm, cl, sh, sm_, sl;
+                    limbs(xc, ch, cm, cl);
+                    limbs(xs, sh, sm_, sl);
+                    const int e = (kb * 32 + gg * 4 + qq) * 4;
+                    frag_w[e + half] = (uint32_t(ch) & 255u) | (uint32_t(cm) & 255u) << 8 | (uint32_t(sh) & 255u) << 16 |
+                                       (uint32_t(sm_) & 255u) << 24;
+                    frag_w[e + 2 + half] = (uint32_t(cm) & 255u) | (uint32_t(cl) & 255u) << 8 | (uint32_t(sm_) & 255u) << 16 |
+                                           (uint32_t(sl) & 255u) << 24;
+                    colx[gg] += double(xc) + double(xs);
+                }
+            }
+        }
+        double *red_d = reinterpret_cast<double *>(off_s + 8);
+#pragma unroll
+        for (int gg = 0; gg < 8; ++gg) {
+            double v = colx[gg];
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+            if ((threadIdx.x & 31) == 0) red_d[8 * (threadIdx.x >> 5) + gg] = v;
+        }
+        __syncthreads();
+        if (threadIdx.x < 8) {
+            double v = 0.0;
+            for (int w = 0; w < WARPS; ++w) v += red_d[8 * w + threadIdx.x];
+            reinterpret_cast<double *>(off_s)[8 * WARPS + threadIdx.x] = 32768.0 * v;   // after the scratch
+        }
+        __syncthreads();
+        return float(1.0 / (double(scale) * double(kI8Sigma)));
     }
     const float scale = pow2_scale(block_max<WARPS>(mx, red_s));  // barriers: sub_s reads are done
     uint32_t *frag_w = reinterpret_cast<uint32_t *>(sm.frag_s);
@@ -1101,8 +1202,9 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 // sincos pair per k-block (measured: N~ = 32 SKA 2140 -> 2186 MVis/s, predict +0.5%; N~ = 24 LOFAR -3.7%,
 // so it is the default for N~ = 32 only).  A one-tile software pipeline of the HMMAs (tried as SCH = 1)
 // compiles to the same SASS as 0: ptxas already spaces the HMMAs 5-12 instructions apart.
-// FX: the A operand split.  1 (default): fixed-point split by byte permutation (split_fx; N~ = 32 SKA loop
-// 7.8 -> 8.8 pairs/clk/SM in scripts/split_probe.cu); 0: the f16 hi/lo split (split2).
+// FX: the A operand.  1: fixed-point f16 split by byte permutation (split_fx; N~ = 32 SKA loop 7.8 -> 8.8
+// pairs/clk/SM against the f16 hi/lo split2 in scripts/split_probe.cu); 2 (the default for 16-row units): the
+// integer form (split_i8, three m16n8k32 u8 x s8 mma per tile into s32 accumulators; R = 8 / 16).
 template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int SCH = 0, int FX = 1>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
@@ -1112,25 +1214,26 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
     const uint4 *frag_s = sm.frag_s;
     const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
     const float *df_s = sm.df_s;
+    static_assert(FX == 1 || (FX == 2 && R >= 8), "A operand form: 1, or 2 with R = 8 / 16 units");
     __shared__ float red_s[WARPS];
-    __shared__ float off_s[FX ? 8 * (WARPS + 1) : 1];
+    __shared__ __align__(16) float off_s[FX == 2 ? 16 * (WARPS + 1) + 8 : 8 * (WARPS + 1)];
 
     const int item = a.order[blockIdx.x];
     const ItemSetup s = dev::item_setup(a, item, NS);
     const idg_metadata &md = s.md;
     const int nc = s.nc;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, q = lane & 3;
-    const float inv0 = degridder_setup_tc<NS, WARPS>(a, s, sm, red_s, FX ? off_s : nullptr);
+    const float inv0 = degridder_setup_tc<NS, WARPS, FX == 2 ? 1 : 0>(a, s, sm, red_s, off_s);
     // output = (acc - off) inv: the fixed-point operand's gain and per-column offset removed
-    const float inv = FX ? inv0 * (1.0f / kFxGain) : inv0;
-    const float off0 = FX ? off_s[2 * q] : 0.0f, off1 = FX ? off_s[2 * q + 1] : 0.0f;
+    const float inv = FX == 1 ? inv0 * (1.0f / kFxGain) : inv0;
+    const float off0 = FX == 1 ? off_s[2 * q] : 0.0f, off1 = FX == 1 ? off_s[2 * q + 1] : 0.0f;
+    const double *offd = reinterpret_cast<const double *>(off_s) + 8 * WARPS;   // FX = 2
+    const double ioff0 = FX == 2 ? offd[2 * q] : 0.0, ioff1 = FX == 2 ? offd[2 * q + 1] : 0.0;
     auto split = [](f2p C, f2p S, uint32_t &hq, uint32_t &lq, uint32_t &hq4, uint32_t &lq4) {
-        if constexpr (FX) {
-            split_fx(C, S, hq, lq, hq4, lq4);
+        if constexpr (FX == 2) {
+            split_i8(C, S, hq, hq4);
         } else {
-            const float2 cc = unpk(C), ss = unpk(S);
-            split_phasor(cc.x, ss.x, hq, lq);
-            split_phasor(cc.y, ss.y, hq4, lq4);
+            split_fx(C, S, hq, lq, hq4, lq4);
         }
     };
 
@@ -1165,15 +1268,23 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
         // row 0 (channel c0) coefficients, and the coefficients of the E phase
         const f2p cu = dup(fmaf(df, cQ.x, cB.x)), cv = dup(fmaf(df, cQ.y, cB.y)), cw = dup(fmaf(df, cQ.z, cB.z));
         const f2p eu = dup(estep * cQ.x), ev = dup(estep * cQ.y), ew = dup(estep * cQ.z);
-        float acc[NTL][4];
+        float acc[FX == 2 ? 1 : NTL][4];
+        int iacc[FX == 2 ? NTL : 1][3][4];   // FX = 2: the s32 sums of the three weight classes
 #pragma unroll
         for (int i = 0; i < NTL; ++i)
 #pragma unroll
-            for (int j = 0; j < 4; ++j) acc[i][j] = 0.0f;
+            for (int j = 0; j < 4; ++j) {
+                if constexpr (FX == 2) {
+                    iacc[i][0][j] = iacc[i][1][j] = iacc[i][2][j] = 0;
+                } else {
+                    acc[i][j] = 0.0f;
+                }
+            }
         static_assert(NKB % UNR == 0, "k-block unroll");
 #pragma unroll UNR
         for (int kb = 0; kb < NKB; ++kb) {
             const uint4 bf = frag_s[kb * 32 + lane];
+            const uint32_t bh0 = FX == 2 ? i8_high_limbs(bf.x) : 0u, bh1 = FX == 2 ? i8_high_limbs(bf.y) : 0u;
             const float4 lm = lmn_s[(kb * 4 + q) * 2], nn = lmn_s[(kb * 4 + q) * 2 + 1];
             const f2p l2 = pk(lm.x, lm.y), m2 = pk(lm.z, lm.w), n2 = pk(nn.x, nn.y);
             const float2 p = unpk(fma2(cu, l2, fma2(cv, m2, mul2(cw, n2))));   // row 0 at slots q, q+4
@@ -1229,8 +1340,13 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                         split(C, S, ah[h2], al[h2], ah[2 + h2], al[2 + h2]);
                         split(C2, S2, bh[h2], bl[h2], bh[2 + h2], bl[2 + h2]);
                     }
-                    mma3(acc[i], ah, al, bf);
-                    mma3(acc[i + H], bh, bl, bf);
+                    if constexpr (FX == 2) {
+                        imma3(iacc[i], ah, bf, bh0, bh1);
+                        imma3(iacc[i + H], bh, bf, bh0, bh1);
+                    } else {
+                        mma3(acc[i], ah, al, bf);
+                        mma3(acc[i + H], bh, bl, bf);
+                    }
                 }
             } else {
                 // R = 8, 16: each tile's three products issued as soon as its two rows are split
@@ -1246,16 +1362,26 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                         }
                         split(C, S, ah[h2], al[h2], ah[2 + h2], al[2 + h2]);
                     }
-                    mma3(acc[i], ah, al, bf);
+                    if constexpr (FX == 2) {
+                        imma3(iacc[i], ah, bf, bh0, bh1);
+                    } else {
+                        mma3(acc[i], ah, al, bf);
+                    }
                 }
             }
         }
         if (valid) {
             float2 *vt = vis0 + int64_t(t) * row + int64_t(c0) * 4 + q;
 #pragma unroll
-            for (int r = 0; r < R; ++r)
-                vt[r * CS * 4] = make_float2((acc[r >> 1][2 * (r & 1)] - off0) * inv,
-                                             (acc[r >> 1][2 * (r & 1) + 1] - off1) * inv);
+            for (int r = 0; r < R; ++r) {
+                if constexpr (FX == 2) {
+                    vt[r * CS * 4] = make_float2(i8_out(iacc[r >> 1], 2 * (r & 1), ioff0, double(inv)),
+                                                 i8_out(iacc[r >> 1], 2 * (r & 1) + 1, ioff1, double(inv)));
+                } else {
+                    vt[r * CS * 4] = make_float2((acc[r >> 1][2 * (r & 1)] - off0) * inv,
+                                                 (acc[r >> 1][2 * (r & 1) + 1] - off1) * inv);
+                }
+            }
         }
     }
 }
@@ -1419,6 +1545,9 @@ const Variant kTcGridder[] = {
 #define TDROTX(NS, W, MB, U, CPT, R, SCH) \
     {NS, CPT, kTensor, 1, "degridder_rot16s" #SCH "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, R, SCH>, CPT, smem_degridder_tc<NS>}
+#define TDROTI(NS, W, MB, U, CPT, R) \
+    {NS, CPT, kTensor, 1, "degridder_rot" #R "i<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, R, 0, 2>, CPT, smem_degridder_tc<NS>}
 #define TDROT(NS, W, MB, U) \
     {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>, 0, \
      smem_degridder_tc<NS>}
@@ -1426,7 +1555,8 @@ const Variant kTcGridder[] = {
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>, 0, \
      smem_degridder_tc<NS>}
 const Variant kTcDegridder[] = {
-    TDROTS(24, 4, 3, 2, 16, 8), TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 2, 32, 16, 2),
+    TDROTS(24, 4, 3, 2, 16, 8), TDROTI(24, 4, 3, 4, 16, 16), TDROTI(32, 4, 2, 4, 32, 16), TDROTI(32, 4, 2, 2, 16, 16),
+    TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 2, 32, 16, 2),
     TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
     TDROTC(24, 8, 2, 1, 8, 8, "degridder_rot8"), TDROTC(32, 16, 2, 1, 8, 8, "degridder_rot8"),
@@ -1439,13 +1569,9 @@ const Variant kTcDegridder[] = {
     // items) -- selected by name only
     TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"),
     TDROTC(24, 8, 2, 1, 16, 8, "degridder_rot8"),
-    // the f16 hi/lo operand split (the default before the fixed-point split), for measurement
-    {24, 16, kTensor, 1, "degridder_rot16f<24,W4,minB3,U4,C16>", launch_degridder_rot<24, 4, 3, 4, 16, 16, 0, 0>, 16,
-     smem_degridder_tc<24>},
-    {32, 32, kTensor, 1, "degridder_rot16s2f<32,W8,minB2,U1,C32>", launch_degridder_rot<32, 8, 2, 1, 32, 16, 2, 0>, 32,
-     smem_degridder_tc<32>},
 };
 #undef TDROTC
+#undef TDROTI
 #undef TDROTS
 #undef TDROTX
 #undef TDROT

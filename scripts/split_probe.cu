@@ -297,6 +297,133 @@ void run8(const char *name, float *out, int ctas_per_sm) {
            pairs / (best * 1e-3) / 148 / 1.965e9, cudaGetErrorString(cudaGetLastError()));
 }
 
+
+// IMMA form: A = 16-bit offset fixed-point phasor as two u8 limbs (one PRMT per phasor: bytes 0, 1 of the
+// (cos, sin) words), B = 24-bit subgrid as three s8 limbs, three m16n8k32 u8 x s8 mma per tile (weights
+// 2^24, 2^16, 2^8) into three s32 accumulators.  R rows per lane, one rotation chain.
+__device__ __forceinline__ void imma(int (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+    asm("mma.sync.aligned.m16n8k32.row.col.s32.u8.s8.s32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, {%0,%1,%2,%3};"
+        : "+r"(d[0]), "+r"(d[1]), "+r"(d[2]), "+r"(d[3]) : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+template <int W, int MINB, int UNR, int R, int CH = 1>
+__global__ void __launch_bounds__(W * 32, MINB) loopi(float *out, int units) {
+    constexpr int NTL = R / 2;
+    extern __shared__ __align__(16) unsigned char smem[];
+    uint4 *frag_s = reinterpret_cast<uint4 *>(smem);      // [NKB][32] {w24, w16}
+    uint2 *frag2_s = reinterpret_cast<uint2 *>(smem + NKB * 32 * 16);   // [NKB][32] {w8}
+    float4 *lmn_s = reinterpret_cast<float4 *>(smem + NKB * 32 * 24);
+    for (int i = threadIdx.x; i < NKB * 32; i += blockDim.x) {
+        frag_s[i] = make_uint4(0x01020304u ^ (i & 0x3ff), 0x05060708u, 0x7f017f01u, 0x11223344u ^ (i & 0xff));
+        frag2_s[i] = make_uint2(0x01020304u ^ i, 0x05060708u);
+    }
+    for (int i = threadIdx.x; i < NKB * 8; i += blockDim.x)
+        lmn_s[i] = make_float4(1e-3f * (i & 31), 2e-3f * (i >> 5), 3e-4f * (i & 7), 1e-4f);
+    __syncthreads();
+    const int lane = threadIdx.x & 31, q = lane & 3;
+    float total = 0.0f;
+    for (int u = 0; u < units * 16 / R; ++u) {
+        const float fu = 0.3f + 1e-3f * u + 1e-4f * lane, fv = 0.2f, fw = 0.05f;
+        const f2p cu = dup(fu), cv = dup(fv), cw = dup(fw);
+        const f2p eu = dup(0.011f), ev = dup(0.007f), ew = dup(0.001f);
+        int acc[NTL][3][4];
+#pragma unroll
+        for (int i = 0; i < NTL; ++i)
+#pragma unroll
+            for (int w = 0; w < 3; ++w)
+#pragma unroll
+                for (int j = 0; j < 4; ++j) acc[i][w][j] = 0;
+#pragma unroll UNR
+        for (int kb = 0; kb < NKB; ++kb) {
+            const uint4 b01 = frag_s[kb * 32 + lane];
+            const uint2 b2 = frag2_s[kb * 32 + lane];
+            const float4 lm = lmn_s[(kb * 4 + q) * 2], nn = lmn_s[(kb * 4 + q) * 2 + 1];
+            const f2p l2 = pk(lm.x, lm.y), m2 = pk(lm.z, lm.w), n2 = pk(nn.x, nn.y);
+            const float2 p = unpk(fma2(cu, l2, fma2(cv, m2, mul2(cw, n2))));
+            const float2 e = unpk(fma2(eu, l2, fma2(ev, m2, mul2(ew, n2))));
+            float s0, c0q, s1, c1q, es0, ec0, es1, ec1;
+            __sincosf(p.x, &s0, &c0q);
+            __sincosf(p.y, &s1, &c1q);
+            __sincosf(e.x, &es0, &ec0);
+            __sincosf(e.y, &es1, &ec1);
+            f2p C = pk(c0q, c1q), S = pk(s0, s1);
+            const f2p EC = pk(ec0, ec1), ES = pk(es0, es1), NES = pk(-es0, -es1);
+            const f2p SIG = dup(32767.0f), MM = dup(8421376.0f);   // 2^23 + 2^15
+            f2p C2 = C, S2 = S;
+            if (CH == 2) {
+                const float2 ph = unpk(fma2(dup(float(R / 2)), pk(e.x, e.y), pk(p.x, p.y)));
+                float sa, ca, sb, cb;
+                __sincosf(ph.x, &sa, &ca);
+                __sincosf(ph.y, &sb, &cb);
+                C2 = pk(ca, cb); S2 = pk(sa, sb);
+            }
+#pragma unroll
+            for (int i = 0; i < NTL / CH; ++i) {
+                uint32_t a[4], b[4];
+#pragma unroll
+                for (int h2 = 0; h2 < 2; ++h2) {
+                    if (i > 0 || h2 > 0) {
+                        const f2p Cn = fma2(C, EC, mul2(S, NES));
+                        S = fma2(C, ES, mul2(S, EC));
+                        C = Cn;
+                        if (CH == 2) {
+                            const f2p Cm = fma2(C2, EC, mul2(S2, NES));
+                            S2 = fma2(C2, ES, mul2(S2, EC));
+                            C2 = Cm;
+                        }
+                    }
+                    const float2 cc = unpk(fma2(C, SIG, MM)), ss = unpk(fma2(S, SIG, MM));
+                    a[h2] = prmt(cc.x, ss.x, 0x5410);
+                    a[2 + h2] = prmt(cc.y, ss.y, 0x5410);
+                    if (CH == 2) {
+                        const float2 cc2 = unpk(fma2(C2, SIG, MM)), ss2 = unpk(fma2(S2, SIG, MM));
+                        b[h2] = prmt(cc2.x, ss2.x, 0x5410);
+                        b[2 + h2] = prmt(cc2.y, ss2.y, 0x5410);
+                    }
+                }
+                imma(acc[i][0], a, b01.x, b01.y);
+                imma(acc[i][1], a, b01.z, b01.w);
+                imma(acc[i][2], a, b2.x, b2.y);
+                if (CH == 2) {
+                    imma(acc[i + NTL / 2][0], b, b01.x, b01.y);
+                    imma(acc[i + NTL / 2][1], b, b01.z, b01.w);
+                    imma(acc[i + NTL / 2][2], b, b2.x, b2.y);
+                }
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < NTL; ++i)
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                total += 16777216.0f * float(acc[i][0][j]) + 65536.0f * float(acc[i][1][j]) + 256.0f * float(acc[i][2][j]);
+    }
+    out[blockIdx.x * blockDim.x + threadIdx.x] = total;
+}
+
+template <int W, int MINB, int UNR, int R, int CH = 1>
+void runi(const char *name, float *out, int ctas_per_sm) {
+    auto k = loopi<W, MINB, UNR, R, CH>;
+    const size_t smem = NKB * 32 * 24 + NKB * 8 * 16;
+    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    cudaFuncAttributes fa;
+    cudaFuncGetAttributes(&fa, k);
+    const int blocks = 148 * ctas_per_sm, units = 40;
+    k<<<blocks, W * 32, smem>>>(out, 2);
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0); cudaEventCreate(&e1);
+    float best = 1e30f;
+    for (int rep = 0; rep < 3; ++rep) {
+        cudaEventRecord(e0);
+        k<<<blocks, W * 32, smem>>>(out, units);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms; cudaEventElapsedTime(&ms, e0, e1);
+        best = ms < best ? ms : best;
+    }
+    const double pairs = double(blocks) * W * units * 128.0 * 1024.0;
+    printf("%-44s regs %3d  %.3f ms  %.2f pairs/clk/SM  %s\n", name, fa.numRegs, best,
+           pairs / (best * 1e-3) / 148 / 1.965e9, cudaGetErrorString(cudaGetLastError()));
+}
+
 // Host check of the byte-permutation split: hi + lo == 3086 + (sigma Z rounded) / 128 exactly.
 __global__ void check(const float *z, float *err, int n) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -329,14 +456,17 @@ int main(int argc, char **argv) {
         for (int i = 0; i < 2 * n; ++i) { mx = fmax(mx, fabs(he[i])); ss += double(he[i]) * he[i]; }
         printf("PRMT split: max |err| %.3e (bound 0.5/sigma = %.3e), rms %.3e\n", mx, 0.5 / kSig, sqrt(ss / (2 * n)));
     }
-    run<1, 8, 2, 1>("VAR1 R16 s2 W8 minB2 U1", out, 2);
-    run8<8, 2, 1, 1>("R8 1 chain W8 minB2 U1", out, 2);
-    run8<8, 2, 2, 1>("R8 1 chain W8 minB2 U2", out, 2);
-    run8<12, 2, 1, 1>("R8 1 chain W12 minB2 U1", out, 2);
-    run8<12, 2, 2, 1>("R8 1 chain W12 minB2 U2", out, 2);
-    run8<8, 2, 1, 2>("R8 2 chains W8 minB2 U1", out, 2);
-    run8<12, 2, 1, 2>("R8 2 chains W12 minB2 U1", out, 2);
-    run8<16, 1, 1, 1>("R8 1 chain W16 minB1 U1", out, 1);
-    run8<16, 1, 2, 1>("R8 1 chain W16 minB1 U2", out, 1);
+    run<1, 8, 2, 2>("VAR1 R16 s2 W8 minB2 U2 (f16 fixed-point)", out, 2);
+    run8<8, 2, 1, 1>("R8 1 chain W8 minB2 U1 (f16 fixed-point)", out, 2);
+    runi<8, 2, 2, 8>("IMMA R8 W8 minB2 U2 (16 warps)", out, 2);
+    runi<8, 2, 1, 8>("IMMA R8 W8 minB2 U1 (16 warps)", out, 2);
+    runi<8, 1, 2, 8>("IMMA R8 W8 minB1 U2 (1 CTA: 8 warps)", out, 1);
+    runi<4, 2, 1, 16>("IMMA R16 W4 minB2 U1 (8 warps)", out, 2);
+    runi<4, 2, 2, 16>("IMMA R16 W4 minB2 U2 (8 warps)", out, 2);
+    runi<4, 2, 1, 16, 2>("IMMA R16 s2 W4 minB2 U1 (8 warps)", out, 2);
+    runi<6, 2, 1, 16>("IMMA R16 W6 minB2 U1 (12 warps)", out, 2);
+    runi<6, 2, 1, 16, 2>("IMMA R16 s2 W6 minB2 U1 (12 warps)", out, 2);
+    runi<8, 1, 1, 16>("IMMA R16 W8 minB1 U1 (8 warps)", out, 1);
+    runi<4, 2, 1, 8>("IMMA R8 W4 minB2 U1 (8 warps)", out, 2);
     return 0;
 }
