@@ -20,6 +20,7 @@ import argparse
 import json
 import math
 import os
+import re
 import statistics
 import sys
 import threading
@@ -211,6 +212,16 @@ STEP_KIND = {"tiny": "grid+degrid", "lofar": "grid+degrid", "lofar_dde": "grid+d
 # e2e: the SKA-shaped set streams from the host as time chunks ("8 time chunks of 1024")
 E2E_TIME_CHUNK = {"ska": 1024}
 TENSOR_FLOPS_PER_PAIR = 96   # split-f16 contraction: 3 products x 16 real MACs x 2 flops per pair
+
+
+def tensor_ops_per_pair(variant: str):
+    """Tensor-core operations executed per (pixel, visibility) pair by a kernel variant: the f16 forms run
+    3 products x 16 real MACs (96 flops); the integer degridders (`degridder_rot16i`) 3 weight classes of
+    m16n8k32 u8 x s8 with 2 limbs per operand value along K (3 x 32 MACs: 192 int8 ops)."""
+    if re.match(r"degridder_rot\d+(s2)?i<", variant or ""):
+        return 192, "3 u8 x s8 weight classes, 2 limbs per value along K"
+    return TENSOR_FLOPS_PER_PAIR, "3 split-f16 products"
+
 
 
 def sincos_per_pair(variant: str, nc_item: int) -> float:
@@ -449,12 +460,15 @@ def run_ours(args):
                 continue
             J = (mjb - mja) / 1e3 / n_e
             sec = e_a.elapsed_time(e_b) * 1e-3 / n_e
-            spp = sincos_per_pair(idg.last_variant(name), nc_item)
+            variant = idg.last_variant(name)
+            spp = sincos_per_pair(variant, nc_item)
+            tops, tdesc = tensor_ops_per_pair(variant)
             per[name] = {"launches": n_e, "J_per_launch": J, "s_per_launch": sec, "avg_W": J / sec,
+                         "variant": variant,
                          "paper_GOps_per_J": OPS_PER_PAIR * pairs / J / 1e9,
-                         "executed_tensor_GFlops_per_J": TENSOR_FLOPS_PER_PAIR * pairs / J / 1e9,
+                         "executed_tensor_GOps_per_J": tops * pairs / J / 1e9,
                          "executed_sincos_G_per_J": spp * pairs / J / 1e9,
-                         "executed": f"per pair: {TENSOR_FLOPS_PER_PAIR} tensor-core flops (3 split-f16 products), "
+                         "executed": f"per pair: {tops} tensor-core ops ({tdesc}), "
                                      f"{spp:g} sincos (MUFU), phasor rotation + operand split on the ALUs"}
         energy["per_kernel"] = per
         energy["paper_context"] = "GTX 1080: 32 / 23 GFlops/W gridder / degridder (P:306; paper-ops: 17 FMA + sincos)"

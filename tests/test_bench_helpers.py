@@ -36,3 +36,10 @@ def test_step_kind_per_config():
     assert bench.STEP_KIND["predict"] == "degrid"                  # configs[4]: degridding-only sweep
     assert all(bench.STEP_KIND[c] == "grid+degrid" for c in ("tiny", "lofar", "lofar_dde", "ska"))
     assert bench.E2E_TIME_CHUNK["ska"] == 1024                      # 8 chunks of 1024
+
+
+def test_tensor_ops_per_pair():
+    from bench import tensor_ops_per_pair as top
+    assert top("degridder_rot16i<32,W4,minB2,U4,C32>")[0] == 192    # integer form: 3 classes x 32 MACs x 2
+    assert top("degridder_rot16<24,W4,minB3,U4,C16>")[0] == 96      # f16 fixed-point split: 3 x 16 x 2
+    assert top("gridder_rot2h<32,W16,MT4,minB2,KPT4,GP4,lmnsm>")[0] == 96

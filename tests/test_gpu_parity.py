@@ -83,6 +83,7 @@ KINDS = {
     "tc": ("tc", "tc"),        # direct tensor-core kernels (one sincos per pair, any channel table)
     "simt": ("simt", "simt"),  # CUDA-core kernels (the paper's structure)
     "umma": ("gridder_umma_rot<*", ""),  # tcgen05 / TMEM rotation gridder, cluster pair (N~ = 32, 16 / 32 ch)
+    "fx16": ("", "degridder_rot16<*"),  # 16-row degridders with the f16 fixed-point split (default: integer form)
 }
 
 
@@ -91,7 +92,7 @@ def kind(request, monkeypatch):
     """Kernel family under test (the variant environment overrides of include/idg.h).  Families a
     case is not eligible for (e.g. tensor-core gridders need C~ % 8 == 0) fall back to the default."""
     g, d = KINDS[request.param]
-    if g:
+    if g or d:
         monkeypatch.setenv("IDG_GRIDDER_VARIANT", g)
         monkeypatch.setenv("IDG_DEGRIDDER_VARIANT", d)
     return request.param
