@@ -1538,10 +1538,11 @@ const Variant kTcGridder[] = {
     {NS, CPT, kTensor, 1, TAG "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, R>, CPT, smem_degridder_tc<NS>}
 // short items (the plan's mean T~ <= 64): 8 channel rows per lane, 4-timestep warp units (finer than the 8 of
-// R = 16, so ragged item tails leave fewer warps idle): lofar_short 3081 -> 3203 MVis/s, LOFAR -7% (r02i)
-#define TDROTS(NS, W, MB, U, CPT, R) \
-    {NS, CPT, kTensor, 1, "degridder_rot8<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
-     launch_degridder_rot<NS, W, MB, U, CPT, R>, CPT, smem_degridder_tc<NS>, 64}
+// R = 16, so ragged item tails leave fewer warps idle): lofar_short 3081 -> 3203 MVis/s, LOFAR -7% (r02i); the
+// integer form (FX = 2) 34.7 -> 33.9 ms on lofar_short (r02zm)
+#define TDROTS(NS, W, MB, U, CPT, R, FX, TAG) \
+    {NS, CPT, kTensor, 1, TAG "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, R, 0, FX>, CPT, smem_degridder_tc<NS>, 64}
 #define TDROTX(NS, W, MB, U, CPT, R, SCH) \
     {NS, CPT, kTensor, 1, "degridder_rot16s" #SCH "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, R, SCH>, CPT, smem_degridder_tc<NS>}
@@ -1555,7 +1556,7 @@ const Variant kTcGridder[] = {
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>, 0, \
      smem_degridder_tc<NS>}
 const Variant kTcDegridder[] = {
-    TDROTS(24, 4, 3, 2, 16, 8), TDROTI(24, 4, 3, 4, 16, 16), TDROTI(32, 4, 2, 4, 32, 16), TDROTI(32, 4, 2, 2, 16, 16),
+    TDROTS(24, 4, 3, 2, 16, 8, 2, "degridder_rot8i"), TDROTI(24, 4, 3, 4, 16, 16), TDROTI(32, 4, 2, 4, 32, 16), TDROTI(32, 4, 2, 2, 16, 16),
     TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 2, 32, 16, 2),
     TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
@@ -1568,7 +1569,7 @@ const Variant kTcDegridder[] = {
     // the single-chain N~ = 32 kernels, and 8-row units for 16-channel items (finer work units for short
     // items) -- selected by name only
     TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"),
-    TDROTC(24, 8, 2, 1, 16, 8, "degridder_rot8"),
+    TDROTC(24, 8, 2, 1, 16, 8, "degridder_rot8"), TDROTS(24, 4, 3, 2, 16, 8, 1, "degridder_rot8"),
 };
 #undef TDROTC
 #undef TDROTI
