@@ -1513,14 +1513,21 @@ cudaError_t launch_degridder_rot(const KernelArgs &a, cudaStream_t st) {
      launch_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM, 1>, 8 * KPT, smem_gridder_rot2<NS, W, MT, MB, KPT, GP, 128, NSM>}
 const Variant kTcGridder[] = {
     TGROT2(24, 12, 3, 2, 2), TGROT2(24, 12, 3, 2, 4), TGROT2(24, 12, 3, 2, 1),
-    TGROT2H(32, 16, 4, 2, 4, 4, 2, "lmnsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"), TGROT2(32, 16, 4, 2, 1),
+    TGROT2H(32, 8, 8, 2, 4, 4, 0, "r"), TGROT2N(32, 8, 8, 2, 2, 2, 0, "r"), TGROT2(32, 16, 4, 2, 1),
     TGROT2(16, 8, 2, 2, 2), TGROT2(16, 8, 2, 2, 4), TGROT2(16, 8, 2, 2, 1),
     TG(24, 12, 3, 2), TG(32, 16, 4, 2), TG(16, 4, 4, 4),
     // alternates kept for measurement (selected by name only): the packed rotation (slower: spills), the
     // E^j form for N~ = 32 (the default before the Horner form), Horner with n only in shared memory.
     // Measured and dropped (r02i / r02o, SKA-T1024, against 135.7 ms): group passes of 1 / 4 in the E^j
-    // form, Horner at 16 warps / SM with 128 registers (138.0), 32 warps of 2 tiles (147.4).
+    // form, Horner at 16 warps x 4 tiles with 128 registers (138.0), 32 warps of 2 tiles (147.4).  Default
+    // since r02zq: 8 warps x 8 tiles at 128 registers (16 warps / SM), pixel coordinates in registers (no
+    // spills): SKA-T1024 136.3 -> 124.7 ms (with lmnsm 130.3; 4 warps x 16 tiles 138.1), predict-T256 (KPT 2)
+    // 251.5 -> 244.0 ms; LOFAR (N~ = 24) keeps 12 warps x 3 tiles (6 x 6: 36.7, 4 x 9: 38.1 against 32.3 ms).
+    // The fixed-point phasor split in the gridders measured 131.7 ms (r02zo) and is not used there.
     TGROT2P(24, 12, 3, 2, 2, 2, 0, "r"), TGROT2N(32, 16, 4, 2, 4, 2, 1, "nsm"), TGROT2H(32, 16, 4, 2, 4, 4, 1, "nsm"),
+    // the defaults before r02zo / r02zq (32 warps x 4 tiles at 64 registers, pixel coordinates re-read from
+    // shared memory to limit the spills)
+    TGROT2H(32, 16, 4, 2, 4, 4, 2, "lmnsm"), TGROT2N(32, 16, 4, 2, 2, 2, 2, "lmnsm"),
     // tcgen05 / TMEM rotation gridder (selected by name while measured)
     GUR(4), GUR(2),
 };
