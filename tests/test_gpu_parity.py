@@ -516,3 +516,26 @@ def test_tolerance_is_discriminating():
     assert err_with(uvw=(obs.uvw * (1 + 2e-5)).astype(np.float32)) > TOL
     assert err_with(v=np.roll(vis, 1, axis=1)) > TOL
     assert err_with(v=vis[..., [0, 2, 1, 3]]) > TOL
+
+
+@pytest.mark.parametrize("name,kw", [("small_dde", {}), ("ska", dict(T=128, nr_stations=4))])
+def test_degrid_amplitude_scaling(name, kw, kind):
+    """The operand forms scale by per-item powers of two, so degrid(2^k G) is exactly 2^k degrid(G)
+    (bitwise) for the fixed-point and integer degridders; a zero grid predicts exact zeros; a grid at
+    1e-20 or 1e+20 amplitude (no power of two) still matches the oracle to the parity bar."""
+    obs = idgsynth.make_observation(name, **kw)
+    _, aterms, tap = _inputs(obs, "random", "asymmetric")
+    G = idgsynth.make_grid(obs)
+    base = gpu_degrid(obs, G, aterms, tap).cpu().numpy()
+    for k in (-40, 37):
+        got = gpu_degrid(obs, (G * np.float32(2.0 ** k)).astype(np.complex64), aterms, tap).cpu().numpy()
+        assert np.array_equal(got, (base * np.float32(2.0 ** k)).astype(np.complex64)), k
+    zero = gpu_degrid(obs, np.zeros_like(G), aterms, tap).cpu().numpy()
+    assert not np.any(zero)
+    items, _ = oracle.plan(obs)
+    for s in (1e-20, 1e20):
+        Gs = (G * s).astype(np.complex64)
+        ref = oracle.scatter_visibilities(obs, items, oracle.degrid(obs, items, Gs, aterms, tap))
+        err = rel_rms(gpu_degrid(obs, Gs, aterms, tap).cpu().numpy(), ref)
+        print(f"degrid[{kind}] {name} amplitude {s:g}: rel rms {err:.3e}")
+        assert err <= TOL, (s, err)
