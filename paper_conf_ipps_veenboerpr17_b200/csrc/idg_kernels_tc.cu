@@ -1594,7 +1594,7 @@ const Variant kTcGridder[] = {
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>, 0, \
      smem_degridder_tc<NS>}
 const Variant kTcDegridder[] = {
-    TDROTS(24, 4, 3, 2, 16, 8, 2, "degridder_rot8i"), TDROTI(24, 4, 3, 4, 16, 16), TDROTI(32, 4, 2, 4, 32, 16), TDROTI(32, 4, 2, 2, 16, 16),
+    TDROTS(24, 4, 3, 2, 16, 8, 2, "degridder_rot8i"), TDROTI(24, 4, 3, 4, 16, 16), TDROTI(32, 4, 2, 4, 32, 16), TDROTI(32, 4, 2, 4, 16, 16),
     TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 2, 32, 16, 2),
     TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
