@@ -938,7 +938,8 @@ struct DegridSmem {
 // over the item's K rows -- the constant the fixed-point A operand adds to every output of column n.
 // BM = 1: the B fragments as the s8 limbs of the integer form (FX = 2) instead: per (k-block, lane)
 // {(x_h, x_m) of slot q, of q+4, (x_m, x_l) of slot q, of q+4}; off_s (16-byte aligned, 16 (WARPS + 1) + 8
-// floats) gets 2^15 sum_k x[k][n] as doubles at double index 8 WARPS + n; returns 1 / (scale sigma).
+// floats) gets 2^15 sum_k x[k][n] as doubles at double index n (the per-warp scratch follows them);
+// returns 1 / (scale sigma).
 template <int NS, int WARPS, int BM = 0>
 __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const ItemSetup &s, const DegridSmem<NS> &sm,
                                                     float *red_s, float *off_s = nullptr) {
@@ -1023,7 +1024,8 @@ __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const I
                 }
             }
         }
-        double *red_d = reinterpret_cast<double *>(off_s + 8);
+        double *offd = reinterpret_cast<double *>(off_s);   // [8] results, then [WARPS][8] scratch
+        double *red_d = offd + 8;
 #pragma unroll
         for (int gg = 0; gg < 8; ++gg) {
             double v = colx[gg];
@@ -1035,7 +1037,7 @@ __device__ __forceinline__ float degridder_setup_tc(const KernelArgs &a, const I
         if (threadIdx.x < 8) {
             double v = 0.0;
             for (int w = 0; w < WARPS; ++w) v += red_d[8 * w + threadIdx.x];
-            reinterpret_cast<double *>(off_s)[8 * WARPS + threadIdx.x] = 32768.0 * v;   // after the scratch
+            offd[threadIdx.x] = 32768.0 * v;
         }
         __syncthreads();
         return float(1.0 / (double(scale) * double(kI8Sigma)));
@@ -1103,7 +1105,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
     const float *df_s = sm.df_s;
     __shared__ float red_s[WARPS];
-    __shared__ __align__(16) float off_s[FX == 2 ? 16 * (WARPS + 1) + 8 : 8 * (WARPS + 1)];
+    __shared__ __align__(16) float off_s[FX == 2 ? 16 * (WARPS + 1) : 8 * (WARPS + 1)];
 
     const int item = a.order[blockIdx.x];
     const ItemSetup s = dev::item_setup(a, item, NS);
@@ -1114,7 +1116,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
     const float inv0 = degridder_setup_tc<NS, WARPS, FX == 2 ? 1 : 0>(a, s, sm, red_s, off_s);
     const float inv = FX == 1 ? inv0 * (1.0f / kFxGain) : inv0;
     const float off0 = FX == 1 ? off_s[2 * q] : 0.0f, off1 = FX == 1 ? off_s[2 * q + 1] : 0.0f;
-    const double *offd = reinterpret_cast<const double *>(off_s) + 8 * WARPS;   // FX = 2
+    const double *offd = reinterpret_cast<const double *>(off_s);   // FX = 2
     const double ioff0 = FX == 2 ? offd[2 * q] : 0.0, ioff1 = FX == 2 ? offd[2 * q + 1] : 0.0;
 
     const int nvis = md.nr_timesteps * nc;
@@ -1244,7 +1246,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
     const float *df_s = sm.df_s;
     static_assert(FX == 1 || (FX == 2 && R >= 8), "A operand form: 1, or 2 with R = 8 / 16 units");
     __shared__ float red_s[WARPS];
-    __shared__ __align__(16) float off_s[FX == 2 ? 16 * (WARPS + 1) + 8 : 8 * (WARPS + 1)];
+    __shared__ __align__(16) float off_s[FX == 2 ? 16 * (WARPS + 1) : 8 * (WARPS + 1)];
 
     const int item = a.order[blockIdx.x];
     const ItemSetup s = dev::item_setup(a, item, NS);
@@ -1255,7 +1257,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
     // output = (acc - off) inv: the fixed-point operand's gain and per-column offset removed
     const float inv = FX == 1 ? inv0 * (1.0f / kFxGain) : inv0;
     const float off0 = FX == 1 ? off_s[2 * q] : 0.0f, off1 = FX == 1 ? off_s[2 * q + 1] : 0.0f;
-    const double *offd = reinterpret_cast<const double *>(off_s) + 8 * WARPS;   // FX = 2
+    const double *offd = reinterpret_cast<const double *>(off_s);   // FX = 2
     const double ioff0 = FX == 2 ? offd[2 * q] : 0.0, ioff1 = FX == 2 ? offd[2 * q + 1] : 0.0;
     auto split = [](f2p C, f2p S, uint32_t &hq, uint32_t &lq, uint32_t &hq4, uint32_t &lq4) {
         if constexpr (FX == 2) {
