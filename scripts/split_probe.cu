@@ -5,8 +5,12 @@
 //          18-bit offset fixed-point Z in the low bits of an fp32 in [2^23, 2^24) whose upper bytes are
 //          the f16 exponent patterns; hi = PRMT(bytes 1, 2), lo = PRMT(bytes 0, 3)            (3 / phasor)
 //   VAR 2  as 1, with the rotation run on W itself (W' = W E + M (1 - E)): no FFMA2 for the split (2 / phasor)
+//   loop8  R = 8 rows per lane with the VAR 1 split, one or two rotation chains
+//   loopi  the integer form: 16-bit fixed-point phasor as two u8 limbs (one PRMT per phasor), three
+//          mma.m16n8k32 u8 x s8 per tile into s32 accumulators (the kernels' degridder_rot16i)
+// VARF bit 4 drops the mma (the ALU side alone), bits 8/16 keep 2 / 1 of the 3 products, bit 32 the rotation.
 // Same shared-memory operands as the kernel (B fragments, slot l/m/n), no global traffic.
-// Prints pairs per clock per SM at the nominal 1965 MHz.
+// Prints pairs per clock per SM at the nominal 1965 MHz (profiles/r02zd_split_probe.txt).
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
