@@ -1600,6 +1600,7 @@ const Variant kTcDegridder[] = {
     TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 2, 32, 16, 2),
     TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
+    TDROTI(24, 8, 2, 1, 8, 8), TDROTI(32, 8, 2, 1, 8, 8), TDROTI(16, 8, 2, 1, 8, 8),   // 8-channel items
     TDROTC(24, 8, 2, 1, 8, 8, "degridder_rot8"), TDROTC(32, 16, 2, 1, 8, 8, "degridder_rot8"),
     TDROTC(16, 8, 2, 1, 8, 8, "degridder_rot8"),
     TDROT(32, 16, 2, 2), TDROT(24, 8, 4, 1), TDROT(16, 8, 4, 1),

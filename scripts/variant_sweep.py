@@ -28,10 +28,12 @@ def main():
     ap.add_argument("--variants", nargs="+", required=True)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=2)
+    ap.add_argument("--obs", nargs="*", default=[], help="extra make_observation keywords, e.g. C=8")
     args = ap.parse_args()
     import torch
     import paper_conf_ipps_veenboerpr17_b200 as idg
-    obs = idgsynth.make_observation(args.config, T=args.timesteps)
+    extra = {k: int(v) for k, v in (kv.split("=") for kv in args.obs)}
+    obs = idgsynth.make_observation(args.config, T=args.timesteps, **extra)
     plan = idg.Plan.from_observation(obs)
     st = plan.stats()
     dev = torch.device("cuda", 0)
