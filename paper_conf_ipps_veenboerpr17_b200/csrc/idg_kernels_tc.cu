@@ -1608,7 +1608,7 @@ const Variant kTcDegridder[] = {
     TDROTC(16, 8, 4, 1, 4, 4, "degridder_rot"),
     // the direct kernel (any channel table) in the integer form (r02zu: LOFAR-T2048 10.35 -> 9.72 ms, SKA-T256
     // 53.6 -> 49.6 ms, parity 3.2e-5 -> 1.4e-5), then in the f16 fixed-point form
-    TDI(24, 8, 2, 3), TDI(32, 8, 2, 2), TD(24, 8, 2, 4), TD(32, 8, 4, 2), TD(16, 8, 4, 2),
+    TDI(24, 8, 2, 3), TDI(32, 8, 2, 2), TDI(16, 8, 2, 2), TD(24, 8, 2, 4), TD(32, 8, 4, 2), TD(16, 8, 4, 2),
     // the single-chain N~ = 32 kernels, and 8-row units for 16-channel items (finer work units for short
     // items) -- selected by name only
     TDROTC(32, 8, 2, 2, 32, 16, "degridder_rot16"), TDROTC(32, 8, 2, 2, 16, 16, "degridder_rot16"),
