@@ -1234,7 +1234,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_tc_kernel(const Ke
 // compiles to the same SASS as 0: ptxas already spaces the HMMAs 5-12 instructions apart.
 // FX: the A operand.  1: fixed-point f16 split by byte permutation (split_fx; N~ = 32 SKA loop 7.8 -> 8.8
 // pairs/clk/SM against the f16 hi/lo split2 in scripts/split_probe.cu); 2 (the default for 16-row units): the
-// integer form (split_i8, three m16n8k32 u8 x s8 mma per tile into s32 accumulators; R = 8 / 16).
+// integer form (split_i8, three m16n8k32 u8 x s8 mma per tile into s32 accumulators).
 template <int NS, int WARPS, int MINB, int UNR, int CPT = 0, int R = 4, int SCH = 0, int FX = 1>
 __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const KernelArgs a) {
     constexpr int NPIX = NS * NS;
@@ -1244,7 +1244,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
     const uint4 *frag_s = sm.frag_s;
     const float4 *lmn_s = sm.lmn_s, *bq_s = sm.bq_s;
     const float *df_s = sm.df_s;
-    static_assert(FX == 1 || (FX == 2 && R >= 8), "A operand form: 1, or 2 with R = 8 / 16 units");
+    static_assert(FX == 1 || FX == 2, "A operand form");
     __shared__ float red_s[WARPS];
     __shared__ __align__(16) float off_s[FX == 2 ? 16 * (WARPS + 1) : 8 * (WARPS + 1)];
 
@@ -1339,12 +1339,17 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) degridder_rot_kernel(const K
                     // tile r >> 1, row g (r even) / g+8 (r odd): A regs {(row, q), (row+8, q), (row, q+4), (row+8, q+4)}
                     split(C, S, ah[r >> 1][r & 1], al[r >> 1][r & 1], ah[r >> 1][2 + (r & 1)], al[r >> 1][2 + (r & 1)]);
                 }
+                if constexpr (FX == 2) {
 #pragma unroll
-                for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
+                    for (int i = 0; i < 2; ++i) imma3(iacc[i], ah[i], bf, bh0, bh1);
+                } else {
 #pragma unroll
-                for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
+                    for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.x, bf.y);
 #pragma unroll
-                for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
+                    for (int i = 0; i < 2; ++i) mma16816(acc[i], ah[i][0], ah[i][1], ah[i][2], ah[i][3], bf.z, bf.w);
+#pragma unroll
+                    for (int i = 0; i < 2; ++i) mma16816(acc[i], al[i][0], al[i][1], al[i][2], al[i][3], bf.x, bf.y);
+                }
             } else if constexpr (SCH == 2) {
                 // R = 8, 16, two rotation chains: tiles i (rows 2i, 2i+1) and i + NTL/2 (rows R/2 + 2i, ...)
                 constexpr int H = NTL / 2;
@@ -1586,6 +1591,9 @@ const Variant kTcGridder[] = {
 #define TDROTI(NS, W, MB, U, CPT, R) \
     {NS, CPT, kTensor, 1, "degridder_rot" #R "i<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, R, 0, 2>, CPT, smem_degridder_tc<NS>}
+#define TDROTI4(NS, W, MB, U, CPT) \
+    {NS, CPT ? CPT : 32, kTensor, 1, "degridder_roti<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
+     launch_degridder_rot<NS, W, MB, U, CPT, 4, 0, 2>, CPT, smem_degridder_tc<NS>}
 #define TDROT(NS, W, MB, U) \
     {NS, 32, kTensor, 1, "degridder_rot<" #NS ",W" #W ",minB" #MB ",U" #U ">", launch_degridder_rot<NS, W, MB, U>, 0, \
      smem_degridder_tc<NS>}
@@ -1603,6 +1611,9 @@ const Variant kTcDegridder[] = {
     TDROTI(24, 8, 2, 1, 8, 8), TDROTI(32, 8, 2, 1, 8, 8), TDROTI(16, 8, 2, 1, 8, 8),   // 8-channel items
     TDROTC(24, 8, 2, 1, 8, 8, "degridder_rot8"), TDROTC(32, 16, 2, 1, 8, 8, "degridder_rot8"),
     TDROTC(16, 8, 2, 1, 8, 8, "degridder_rot8"),
+    // 4-row units (C~ a multiple of 32 other than 32; 4 channels): integer form, then the f16 fixed-point form
+    TDROTI4(32, 8, 2, 2, 0), TDROTI4(24, 8, 3, 1, 0), TDROTI4(16, 8, 3, 1, 0),
+    TDROTI4(24, 8, 3, 1, 4), TDROTI4(32, 8, 2, 1, 4), TDROTI4(16, 8, 3, 1, 4),
     TDROT(32, 16, 2, 2), TDROT(24, 8, 4, 1), TDROT(16, 8, 4, 1),
     TDROTC(24, 8, 4, 1, 4, 4, "degridder_rot"), TDROTC(32, 16, 2, 1, 4, 4, "degridder_rot"),
     TDROTC(16, 8, 4, 1, 4, 4, "degridder_rot"),
@@ -1616,6 +1627,7 @@ const Variant kTcDegridder[] = {
 };
 #undef TDROTC
 #undef TDROTI
+#undef TDROTI4
 #undef TDI
 #undef TDROTS
 #undef TDROTX
