@@ -217,8 +217,9 @@ TENSOR_FLOPS_PER_PAIR = 96   # split-f16 contraction: 3 products x 16 real MACs 
 def tensor_ops_per_pair(variant: str):
     """Tensor-core operations executed per (pixel, visibility) pair by a kernel variant: the f16 forms run
     3 products x 16 real MACs (96 flops); the integer degridders (`degridder_rot16i`) 3 weight classes of
-    m16n8k32 u8 x s8 with 2 limbs per operand value along K (3 x 32 MACs: 192 int8 ops)."""
-    if re.match(r"degridder_rot\d+(s2)?i<", variant or ""):
+    m16n8k32 u8 x s8 with 2 limbs per operand value along K (3 x 32 MACs: 192 int8 ops); likewise the
+    integer 8- / 4-row units (`rot8i`, `roti`) and the integer direct kernel (`degridder_tci`)."""
+    if re.match(r"degridder_(rot\d*(s2)?|tc)i<", variant or ""):
         return 192, "3 u8 x s8 weight classes, 2 limbs per value along K"
     return TENSOR_FLOPS_PER_PAIR, "3 split-f16 products"
 

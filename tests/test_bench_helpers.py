@@ -42,4 +42,7 @@ def test_tensor_ops_per_pair():
     from bench import tensor_ops_per_pair as top
     assert top("degridder_rot16i<32,W4,minB2,U4,C32>")[0] == 192    # integer form: 3 classes x 32 MACs x 2
     assert top("degridder_rot16<24,W4,minB3,U4,C16>")[0] == 96      # f16 fixed-point split: 3 x 16 x 2
+    for name in ("degridder_roti<24,W8,minB3,U1,C4>", "degridder_rot8i<24,W4,minB3,U2,C16>", "degridder_tci<32,W8,MT2,minB2>"):
+        assert top(name)[0] == 192, name
+    assert top("degridder_tc<32,W8,MT4,minB2>")[0] == 96
     assert top("gridder_rot2h<32,W16,MT4,minB2,KPT4,GP4,lmnsm>")[0] == 96
