@@ -1604,7 +1604,9 @@ const Variant kTcGridder[] = {
     {NS, 0, kTensor, 0, "degridder_tc<" #NS ",W" #W ",MT" #MT ",minB" #MB ">", launch_degridder_tc<NS, W, MT, MB>, 0, \
      smem_degridder_tc<NS>}
 const Variant kTcDegridder[] = {
-    TDROTS(24, 4, 3, 2, 16, 8, 2, "degridder_rot8i"), TDROTI(24, 4, 3, 4, 16, 16), TDROTI(32, 4, 2, 4, 32, 16), TDROTI(32, 4, 2, 4, 16, 16),
+    // 16-row integer units at k-block unroll 8 (r02zz: against U4 SKA-T1024 140.7 -> 138.8 ms, predict-T256
+    // 214.2 -> 212.1, LOFAR 27.53 -> 27.30)
+    TDROTS(24, 4, 3, 2, 16, 8, 2, "degridder_rot8i"), TDROTI(24, 4, 3, 8, 16, 16), TDROTI(32, 4, 2, 8, 32, 16), TDROTI(32, 4, 2, 8, 16, 16),
     TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 2, 32, 16, 2),
     TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
