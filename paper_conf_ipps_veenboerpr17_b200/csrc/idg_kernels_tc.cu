@@ -1581,7 +1581,7 @@ const Variant kTcGridder[] = {
      launch_degridder_rot<NS, W, MB, U, CPT, R>, CPT, smem_degridder_tc<NS>}
 // short items (the plan's mean T~ <= 64): 8 channel rows per lane, 4-timestep warp units (finer than the 8 of
 // R = 16, so ragged item tails leave fewer warps idle): lofar_short 3081 -> 3203 MVis/s, LOFAR -7% (r02i); the
-// integer form (FX = 2) 34.7 -> 33.9 ms on lofar_short (r02zm)
+// integer form (FX = 2) 34.7 -> 33.9 ms on lofar_short (r02zm), at unroll 4 33.1 ms (r02zz)
 #define TDROTS(NS, W, MB, U, CPT, R, FX, TAG) \
     {NS, CPT, kTensor, 1, TAG "<" #NS ",W" #W ",minB" #MB ",U" #U ",C" #CPT ">", \
      launch_degridder_rot<NS, W, MB, U, CPT, R, 0, FX>, CPT, smem_degridder_tc<NS>, 64}
@@ -1606,7 +1606,7 @@ const Variant kTcGridder[] = {
 const Variant kTcDegridder[] = {
     // 16-row integer units at k-block unroll 8 (r02zz: against U4 SKA-T1024 140.7 -> 138.8 ms, predict-T256
     // 214.2 -> 212.1, LOFAR 27.53 -> 27.30)
-    TDROTS(24, 4, 3, 2, 16, 8, 2, "degridder_rot8i"), TDROTI(24, 4, 3, 8, 16, 16), TDROTI(32, 4, 2, 8, 32, 16), TDROTI(32, 4, 2, 8, 16, 16),
+    TDROTS(24, 4, 3, 4, 16, 8, 2, "degridder_rot8i"), TDROTI(24, 4, 3, 8, 16, 16), TDROTI(32, 4, 2, 8, 32, 16), TDROTI(32, 4, 2, 8, 16, 16),
     TDROTC(24, 4, 3, 4, 16, 16, "degridder_rot16"), TDROTX(32, 8, 2, 2, 32, 16, 2),
     TDROTX(32, 8, 2, 1, 16, 16, 2), TDROTC(16, 8, 2, 1, 16, 16, "degridder_rot16"),
     TDROTC(16, 8, 2, 1, 32, 16, "degridder_rot16"),
